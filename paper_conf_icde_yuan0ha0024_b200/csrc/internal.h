@@ -1,0 +1,127 @@
+// Internal declarations of libtdfs.so (not part of the ABI).
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "tdfs.h"
+
+namespace tdfs {
+
+constexpr int kMaxK = TDFS_MAX_K;
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+int fail(int status, const std::string& msg);  // sets the detail, returns status
+
+// ---------------------------------------------------------------- plan
+// Per matching-order position p (pi_p = order[p]) everything the kernel needs,
+// precomputed on the host (PAPER.md:77 backward neighbours, :29 constraints,
+// :400 degree/label filters).  Bit j of a mask refers to position j < p.
+struct DevPlan {
+  int32_t k;
+  int32_t order[kMaxK];      // query vertex at position p (enumerate output mapping)
+  uint32_t bwd[kMaxK];       // B^pi(pi_p) as a position mask
+  uint32_t lo_mask[kMaxK];   // j with constraint f(pi_j) < f(pi_p): v > S[j]
+  uint32_t hi_mask[kMaxK];   // j with constraint f(pi_p) < f(pi_j): v < S[j]
+  uint32_t inj_mask[kMaxK];  // j whose v != S[j] is not implied by adjacency or a constraint
+  int32_t label[kMaxK];      // required label, -1 = any
+  int32_t deg_min[kMaxK];    // degree filter threshold (0 = off), R8
+  int32_t edge_cons;         // constraint between positions 0 and 1: +1 S0<S1, -1 S1<S0, 0 none
+  int32_t pad_;
+};
+
+struct Plan {
+  int k = 0;
+  std::vector<std::pair<int, int>> qedges;
+  std::vector<int> qlabel;   // empty = unlabeled
+  std::vector<int> order;
+  std::vector<std::pair<int, int>> constraints;
+  int64_t n_aut = 1;
+  DevPlan dev{};
+};
+
+// ---------------------------------------------------------------- graph
+struct Graph {
+  int device = 0;
+  int64_t n = 0, nnz = 0, dmax = 0;
+  int32_t nlabels = 1;
+  int64_t* d_offs = nullptr;
+  int32_t* d_adj = nullptr;
+  uint8_t* d_label = nullptr;
+  int32_t* d_src = nullptr;  // source vertex of each directed entry (edge tasks)
+  bool owns_csr = true;
+};
+
+// ---------------------------------------------------------------- device job
+struct QSlot {                // one task of Q_task, 16 bytes (PAPER.md:191 uses 3 ints)
+  int32_t v1, v2, v3;
+  uint32_t seq;               // ticket handshake: == t free for ticket t, == t+1 full for ticket t
+};
+
+enum CounterIdx {            // each counter on its own 128-byte line
+  C_COUNT = 0, C_CURSOR, C_QHEAD, C_QTAIL, C_QAVAIL, C_QFREE, C_ACTIVE, C_POOL, C_ERROR, C_OUTCUR, C_TRACE,
+  C_NUM
+};
+constexpr int kCounterStride = 16;  // u64 words per counter (128 B)
+
+enum StatIdx {
+  S_NODES = 0,                 // 9 entries
+  S_ADJ_BYTES = 9, S_ENQ, S_DEQ, S_TIMEOUTS, S_QFULL, S_EDGES_SCANNED, S_EDGES_IN, S_CHUNKS,
+  S_NUM
+};
+
+struct KParams {
+  // graph
+  const int64_t* offs;
+  const int32_t* adj;
+  const int32_t* src;
+  const uint8_t* label;
+  int64_t n;
+  // plan
+  DevPlan plan;
+  // initial tasks: this shard's directed edges e = shard_rank + j * shard_world
+  int64_t n_tasks;             // number of j
+  int32_t shard_rank, shard_world;
+  int32_t chunk;
+  int32_t n_levels;            // stored stack levels = max(0, k - 3): positions 2 .. k-2
+  // queue
+  QSlot* slots;
+  uint64_t qcap;
+  // counters
+  unsigned long long* ctr;     // C_NUM * kCounterStride u64
+  unsigned long long* stats;   // S_NUM u64 or nullptr
+  // paged stacks (Alg. 5)
+  uint32_t* page_tables;       // [n_warps][n_levels][E], 0xFFFFFFFF = null
+  int32_t* pool;               // n_pages pages of (1 << page_shift) ints
+  uint32_t n_pages;
+  int32_t page_shift;          // log2(ints per page)
+  int32_t E;                   // page-table entries per level
+  int64_t tau_ns;              // < 0: infinity
+  // enumerate
+  int32_t* out;
+  unsigned long long cap;
+  // tracing (tests)
+  int32_t* trace;
+  long long trace_cap;
+};
+
+// workspace layout (byte offsets from the 256-aligned base)
+struct WsLayout {
+  size_t ctr = 0, stats = 0, slots = 0, tables = 0, pool = 0, total = 0;
+  uint64_t qcap = 0, n_pages = 0;
+  int32_t E = 0, page_shift = 0, n_levels = 0, blocks = 0, wpb = 0;
+};
+
+int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayout* L);
+int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
+               int mode /*0 count, 1 enumerate*/, int32_t* d_out, uint64_t cap, uint64_t* d_count,
+               bool sync, uint64_t* h_count, tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap,
+               int64_t* n_trace);
+int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int* out);
+const Graph* graph_of(const tdfs_graph* g);
+const Plan* plan_of(const tdfs_plan* p);
+
+}  // namespace tdfs

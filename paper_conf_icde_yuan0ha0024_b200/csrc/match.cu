@@ -1,0 +1,665 @@
+// The T-DFS hot path on sm_100a: one persistent kernel per job.
+//
+// Per warp (the basic processing unit):
+//   outer loop   take a task from Q_task first (Alg. 4 l.1-3), else the
+//                next chunk of initial edge tasks of this GPU's shard (l.4-5,
+//                PAPER.md:122), edge-filtered in the warp; exit when
+//                no work remains anywhere (termination rule, R12).
+//   DFS          iterative backtracking over matching-order positions with per-level
+//                size/iter (Alg. 2 / Alg. 4); S, size[],
+//                iter[] live in lane-indexed registers (lane p holds position p).
+//   timeout      before descending at a split-eligible level (task prefix <= 3
+//                matched vertices) lane 0 reads %globaltimer; when
+//                now - t0 >= tau the current and all remaining siblings are pushed to
+//                Q_task and the warp backtracks (Alg. 4 l.12-21);
+//                a full queue resets t0 (l.18-20).
+//   stacks       each stored level is a page table over fixed-size pages taken from a
+//                device pool on first touch and kept for the whole job (Alg. 5,
+//                PAPER.md:340-390); a batch of <= 32 outputs crosses <= 1 page
+//                boundary; allocation is warp-uniform (lane 0), so no
+//                divergent leader election is needed.  Exhaustion is an error, never a
+//                truncated count.
+//   Eq. (1)      candidates = intersection of the backward neighbours' sorted
+//                adjacency lists, computed warp-cooperatively: the
+//                shortest operand is streamed with coalesced loads, one element per
+//                lane, and each other operand is probed by per-lane binary search
+//                whose lower bound advances batch by batch;
+//                symmetry-breaking constraints become a [lo, hi) id window applied by
+//                binary search before the scan; injectivity,
+//                label and degree filters are fused; survivors are
+//                compacted with __ballot_sync/__popc into the next level, or only
+//                counted at the last level.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstring>
+
+#include "internal.h"
+
+namespace tdfs {
+namespace {
+
+#include "prims.cuh"
+
+// ------------------------------------------------------------ warp context
+template <bool STATS>
+struct Ctx {
+  int lane;
+  int sreg;                 // lane p: S[p]
+  long long lsize, liter;   // lane p: size[p], iter[p]
+  unsigned long long count;  // warp-uniform
+  unsigned long long t0;     // lane 0: task start time
+  unsigned long long lnodes; // lane p: nodes[p]   (STATS)
+  unsigned long long wbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
+  uint32_t* tables;         // this warp's page tables [n_levels][E]
+};
+
+__device__ __forceinline__ int getS(int sreg, int p) { return __shfl_sync(FULL, sreg, p); }
+
+// timeout test (lane 0 decides, broadcast)
+template <bool STATS>
+__device__ __forceinline__ bool timed_out(const KParams& P, Ctx<STATS>& c) {
+  if (P.tau_ns < 0) return false;
+  int t = 0;
+  if (c.lane == 0) t = (long long)(globaltimer() - c.t0) >= P.tau_ns;
+  return __shfl_sync(FULL, t, 0) != 0;
+}
+
+// Candidate generation for position d (Eq. 1 + fused filters).
+// MODE_OUT: 0 = store into the paged level of d; 1 = count only (last position);
+//           2 = enumerate (last position).
+// Returns the number of candidates, or -1 on stack exhaustion.
+template <int MODE_OUT, bool STATS>
+__device__ long long extend(const KParams& P, Ctx<STATS>& c, int d) {
+  const int lane = c.lane;
+  const DevPlan& pl = P.plan;
+  const uint32_t bm = pl.bwd[d];
+  const int nops = __popc(bm);
+  // operand t (lane t < nops) = adjacency list of S[j_t], j_t = t-th set bit of bm
+  int jt = 0;
+  {
+    uint32_t m = bm;
+    for (int i = 0; i < lane && m; i++) m &= m - 1;
+    jt = m ? (__ffs(m) - 1) : 0;
+  }
+  int sj = __shfl_sync(FULL, c.sreg, jt);
+  long long ob = 0, oe = 0;
+  if (lane < nops) {
+    ob = __ldg(P.offs + sj);
+    oe = __ldg(P.offs + sj + 1);
+  }
+  if (STATS) {
+    unsigned long long wb = (lane < nops) ? (unsigned long long)(4 * (oe - ob) + 16) : 0ull;
+    for (int o = 16; o > 0; o >>= 1) wb += __shfl_xor_sync(FULL, wb, o);
+    if (lane == 0) c.wbytes += wb;
+  }
+  // constraint window [lo, hi)
+  const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
+  int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
+  int hi = __reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
+  if (lo >= hi) return 0;
+  if (lane < nops && (lo > 0 || hi < INT_MAX)) {
+    const int32_t* L = P.adj + ob;
+    int n = (int)(oe - ob);
+    int a = lo > 0 ? lower_bound_dev(L, n, lo) : 0;
+    int b = hi < INT_MAX ? a + lower_bound_dev(L + a, n - a, hi) : n;
+    oe = ob + b;
+    ob = ob + a;
+  }
+  long long len = (lane < nops) ? (oe - ob) : LLONG_MAX;
+  // shortest operand
+  unsigned minlen = __reduce_min_sync(FULL, (unsigned)min(len, (long long)UINT_MAX));
+  if (minlen == 0) return 0;
+  int tA = __ffs(__ballot_sync(FULL, lane < nops && (unsigned)len == minlen)) - 1;
+  const long long bA = __shfl_sync(FULL, ob, tA);
+  const long long eA = __shfl_sync(FULL, oe, tA);
+  const uint32_t others = __ballot_sync(FULL, lane < nops && lane != tA);
+  const uint32_t injm = pl.inj_mask[d];
+  const int need_label = pl.label[d];
+  const int dmin = pl.deg_min[d];
+
+  PagedWriter w;
+  w.table = c.tables + (size_t)(d - 2) * P.E;
+  w.cur_p = -1;
+  w.cur_pg = NULL_PAGE;
+  long long total = 0;
+
+  for (long long base = bA; base < eA; base += 32) {
+    const long long i = base + lane;
+    const bool inr = i < eA;
+    const int v = inr ? __ldg(P.adj + i) : INT_MAX;
+    bool ok = inr;
+    const int last_lane = (int)min(31ll, eA - 1 - base);
+    // probe the other operands (per-lane binary search, advancing lower bound)
+    uint32_t om = others;
+    while (om) {
+      const int t = __ffs(om) - 1;
+      om &= om - 1;
+      const long long tb = __shfl_sync(FULL, ob, t);
+      const long long te = __shfl_sync(FULL, oe, t);
+      int pos = (int)(te - tb);
+      const bool probe = inr && (ok || lane == last_lane);
+      if (probe) pos = lower_bound_dev(P.adj + tb, (int)(te - tb), v);
+      if (ok) ok = (pos < te - tb) && __ldg(P.adj + tb + pos) == v;
+      const int adv = __shfl_sync(FULL, pos, last_lane);
+      if (lane == t) ob = tb + adv;
+      if (!__any_sync(FULL, ok)) break;
+    }
+    // fused filters: injectivity, label, degree
+    if (injm) {
+      uint32_t m = injm;
+      while (m) {
+        const int j = __ffs(m) - 1;
+        m &= m - 1;
+        const int s = getS(c.sreg, j);
+        ok = ok && (v != s);
+      }
+    }
+    if (need_label >= 0 && ok) ok = (P.label ? (int)__ldg(P.label + v) : 0) == need_label;
+    if (dmin > 0 && ok) ok = (__ldg(P.offs + v + 1) - __ldg(P.offs + v)) >= dmin;
+    const unsigned bal = __ballot_sync(FULL, ok);
+    const int cnt = __popc(bal);
+    if (MODE_OUT == 0) {
+      if (!paged_write(P, w, bal, total, v, lane)) return -1;
+    } else if (MODE_OUT == 2 && cnt) {
+      unsigned long long ob0 = 0;
+      if (lane == 0) ob0 = atomicAdd(ctr(P, C_OUTCUR), (unsigned long long)cnt);
+      ob0 = __shfl_sync(FULL, ob0, 0);
+      const int k = pl.k;
+      const unsigned long long idx = ob0 + __popc(bal & lanemask_lt());
+      for (int p = 0; p < k - 1; p++) {
+        const int s = getS(c.sreg, p);
+        if (ok && idx < P.cap) P.out[idx * k + pl.order[p]] = s;
+      }
+      if (ok && idx < P.cap) P.out[idx * k + pl.order[k - 1]] = v;
+    }
+    total += cnt;
+  }
+  if (STATS && lane == d) c.lnodes += (unsigned long long)total;
+  return total;
+}
+
+// Push <S0, S1, L[2][i]> for i in [from, size) -- timeout split of level 2
+// (PAPER.md:268).  Returns the first index NOT pushed (size on success).
+template <bool STATS>
+__device__ long long split_level2(const KParams& P, Ctx<STATS>& c, const Queue& q, long long from, long long size) {
+  const uint32_t* table = c.tables;  // level index 0 = position 2
+  const int s0 = getS(c.sreg, 0), s1 = getS(c.sreg, 1);
+  for (long long base = from; base < size; base += 32) {
+    const long long i = base + c.lane;
+    int v = 0;
+    if (i < size) v = paged_read(P, table, i);
+    const unsigned mask = __ballot_sync(FULL, i < size);
+    if (!q_push_warp(P, q, mask, s0, s1, v, c.lane)) {
+      if (STATS && c.lane == 0) c.qfull++;
+      return base;
+    }
+    if (STATS && c.lane == 0) c.enq += __popc(mask);
+  }
+  return size;
+}
+
+// Depth-first search below a prefix S[0..start-1] (Alg. 4 l.7-28).
+// Returns false on error.
+template <int MODE, bool STATS>
+__device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) {
+  const int k = P.plan.k;
+  const int lane = c.lane;
+  if (start == k - 1) {
+    long long n = (MODE == 1) ? extend<2, STATS>(P, c, start) : extend<1, STATS>(P, c, start);
+    c.count += (unsigned long long)n;
+    return true;
+  }
+  int d = start;
+  long long sz = extend<0, STATS>(P, c, d);
+  if (sz < 0) return false;
+  if (lane == d) { c.lsize = sz; c.liter = 0; }
+  for (;;) {
+    const long long it = __shfl_sync(FULL, c.liter, d);
+    const long long size = __shfl_sync(FULL, c.lsize, d);
+    if (it < size) {
+      if (d == 2 && timed_out(P, c)) {
+        // timeout: push the current and all remaining siblings, then backtrack
+        if (STATS && lane == 0) c.touts++;
+        long long upto = split_level2(P, c, q, it, size);
+        if (upto >= size) {
+          if (lane == d) c.liter = size;
+          continue;
+        }
+        // queue full: the pushed prefix is gone, continue in place with t0 reset
+        if (lane == d) c.liter = upto;
+        if (lane == 0) c.t0 = globaltimer();
+        continue;
+      }
+      const uint32_t* table = c.tables + (size_t)(d - 2) * P.E;
+      const int v = paged_read(P, table, it);
+      if (lane == d) { c.sreg = v; c.liter = it + 1; }
+      if (d + 1 == k - 1) {
+        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1) : extend<1, STATS>(P, c, d + 1);
+        c.count += (unsigned long long)n;
+      } else {
+        d++;
+        sz = extend<0, STATS>(P, c, d);
+        if (sz < 0) return false;
+        if (lane == d) { c.lsize = sz; c.liter = 0; }
+      }
+    } else {
+      if (d == start) break;
+      d--;
+    }
+  }
+  return true;
+}
+
+// Process one chunk [j0, j1) of this shard's directed edges (Alg. 4 l.5, edge
+// filtering PAPER.md:400).  Returns false on error.
+template <int MODE, bool STATS>
+__device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long long j0, long long j1) {
+  const int lane = c.lane;
+  const DevPlan& pl = P.plan;
+  const int k = pl.k;
+  for (long long jb = j0; jb < j1; jb += 32) {
+    const long long j = jb + lane;
+    const bool inr = j < j1;
+    int v0 = 0, v1 = 0;
+    bool ok = inr;
+    if (inr) {
+      const long long e = (long long)P.shard_rank + j * (long long)P.shard_world;
+      v0 = __ldg(P.src + e);
+      v1 = __ldg(P.adj + e);
+      if (pl.edge_cons == 1) ok = v0 < v1;
+      else if (pl.edge_cons == -1) ok = v1 < v0;
+      else if (pl.edge_cons == 2) ok = false;
+      if (ok && pl.label[0] >= 0) ok = (P.label ? (int)__ldg(P.label + v0) : 0) == pl.label[0];
+      if (ok && pl.label[1] >= 0) ok = (P.label ? (int)__ldg(P.label + v1) : 0) == pl.label[1];
+      if (ok && pl.deg_min[0] > 1) ok = (__ldg(P.offs + v0 + 1) - __ldg(P.offs + v0)) >= pl.deg_min[0];
+      if (ok && pl.deg_min[1] > 1) ok = (__ldg(P.offs + v1 + 1) - __ldg(P.offs + v1)) >= pl.deg_min[1];
+    }
+    unsigned mask = __ballot_sync(FULL, ok);
+    if (STATS) {
+      if (lane == 1) c.lnodes += __popc(mask);
+      if (lane == 0) {
+        c.scanned += __popc(__ballot_sync(FULL, inr));
+        c.edges_in += __popc(mask);
+      }
+    } else {
+      (void)0;
+    }
+    if (k == 2) {  // the query is one edge: every filtered edge is a match
+      const int cnt = __popc(mask);
+      if (MODE == 1 && cnt) {
+        unsigned long long ob0 = 0;
+        if (lane == 0) ob0 = atomicAdd(ctr(P, C_OUTCUR), (unsigned long long)cnt);
+        ob0 = __shfl_sync(FULL, ob0, 0);
+        const unsigned long long idx = ob0 + __popc(mask & lanemask_lt());
+        if (ok && idx < P.cap) {
+          P.out[idx * 2 + pl.order[0]] = v0;
+          P.out[idx * 2 + pl.order[1]] = v1;
+        }
+      }
+      c.count += (unsigned long long)cnt;
+      continue;
+    }
+    while (mask) {
+      // timeout check before descending into the next edge (edge level is split-eligible)
+      if (timed_out(P, c)) {
+        if (STATS && lane == 0) c.touts++;
+        if (q_push_warp(P, q, mask, v0, v1, -2, lane)) {
+          if (STATS && lane == 0) c.enq += __popc(mask);
+          mask = 0;
+          break;
+        }
+        if (STATS && lane == 0) c.qfull++;
+        if (lane == 0) c.t0 = globaltimer();
+      }
+      const int l = __ffs(mask) - 1;
+      mask &= mask - 1;
+      const int a = __shfl_sync(FULL, v0, l), b = __shfl_sync(FULL, v1, l);
+      if (lane == 0) c.sreg = a;
+      if (lane == 1) c.sreg = b;
+      if (!dfs<MODE, STATS>(P, c, q, 2)) return false;
+    }
+    if (read_error(P)) return false;
+  }
+  return true;
+}
+
+// The persistent matching kernel.  MODE 0 = count, 1 = enumerate.
+template <int MODE, bool STATS>
+__global__ void __launch_bounds__(128, 8) tdfs_kernel(const KParams P) {
+  const int lane = threadIdx.x & 31;
+  const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  Ctx<STATS> c;
+  c.lane = lane;
+  c.sreg = -1;
+  c.lsize = 0;
+  c.liter = 0;
+  c.count = 0;
+  c.t0 = 0;
+  c.lnodes = 0;
+  c.wbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
+  c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
+  const Queue q = make_queue(P);
+  int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
+  unsigned long long* cursor = ctr(P, C_CURSOR);
+
+  if (lane == 0) atomicAdd(active, 1);
+  bool busy = true;
+  for (;;) {
+    if (read_error(P)) break;
+    if (!busy) {
+      // idle: wait for queued tasks; exit when no warp is busy and the queue is empty
+      int go = 0;
+      if (lane == 0) {
+        if (ld_relaxed_s64(q.avail) > 0) {
+          atomicAdd(active, 1);
+          go = 1;
+        } else {
+          __threadfence();
+          go = (ld_relaxed_s32(active) == 0) ? -1 : 0;
+        }
+      }
+      go = __shfl_sync(FULL, go, 0);
+      if (go < 0) break;
+      if (go == 0) {
+        __nanosleep(256);
+        continue;
+      }
+      busy = true;
+    }
+    // 1. Q_task first
+    int got = 0, t1 = 0, t2 = 0, t3 = 0;
+    if (lane == 0) {
+      got = q_pop(q, t1, t2, t3);
+      if (got) c.t0 = globaltimer();
+    }
+    got = __shfl_sync(FULL, got, 0);
+    if (got) {
+      t1 = __shfl_sync(FULL, t1, 0);
+      t2 = __shfl_sync(FULL, t2, 0);
+      t3 = __shfl_sync(FULL, t3, 0);
+      if (STATS && lane == 0) c.deq++;
+      if (lane == 0) c.sreg = t1;
+      if (lane == 1) c.sreg = t2;
+      if (lane == 2) c.sreg = t3;
+      if (!dfs<MODE, STATS>(P, c, q, t3 == -2 ? 2 : 3)) {
+        raise_error(P, ERR_STACK);
+        break;
+      }
+      continue;
+    }
+    // 2. next chunk of initial edge tasks
+    long long j0 = P.n_tasks;
+    if (lane == 0) {
+      if ((long long)ld_relaxed_s64(cursor) < P.n_tasks) {
+        j0 = (long long)atomicAdd(cursor, (unsigned long long)P.chunk);
+        c.t0 = globaltimer();
+      }
+    }
+    j0 = __shfl_sync(FULL, j0, 0);
+    if (j0 < P.n_tasks) {
+      if (STATS && lane == 0) c.chunks++;
+      long long j1 = min(j0 + (long long)P.chunk, (long long)P.n_tasks);
+      if (!run_chunk<MODE, STATS>(P, c, q, j0, j1)) {
+        raise_error(P, ERR_STACK);
+        break;
+      }
+      continue;
+    }
+    // 3. nothing to do: become idle
+    if (lane == 0) {
+      __threadfence();
+      atomicSub(active, 1);
+    }
+    busy = false;
+  }
+  if (busy && lane == 0) atomicSub(active, 1);
+  // publish this warp's results
+  if (lane == 0 && c.count) atomicAdd(ctr(P, C_COUNT), c.count);
+  if (STATS && P.stats) {
+    if (lane < kMaxK + 1 && c.lnodes) atomicAdd(P.stats + S_NODES + lane, c.lnodes);
+    if (lane == 0) {
+      atomicAdd(P.stats + S_ADJ_BYTES, c.wbytes);
+      atomicAdd(P.stats + S_ENQ, c.enq);
+      atomicAdd(P.stats + S_DEQ, c.deq);
+      atomicAdd(P.stats + S_TIMEOUTS, c.touts);
+      atomicAdd(P.stats + S_QFULL, c.qfull);
+      atomicAdd(P.stats + S_EDGES_SCANNED, c.scanned);
+      atomicAdd(P.stats + S_EDGES_IN, c.edges_in);
+      atomicAdd(P.stats + S_CHUNKS, c.chunks);
+    }
+  }
+}
+
+// Initialise the queue's per-slot sequence words for ticket base `base`.
+__global__ void init_queue_kernel(QSlot* slots, unsigned long long cap, unsigned long long base) {
+  for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < cap;
+       s += (unsigned long long)gridDim.x * blockDim.x) {
+    unsigned long long first = base + ((s + cap - (base % cap)) % cap);  // first ticket >= base hitting slot s
+    slots[s].seq = (unsigned)first;
+    slots[s].v1 = slots[s].v2 = slots[s].v3 = -1;
+  }
+}
+
+__global__ void init_counters_kernel(unsigned long long* ctrs, unsigned long long qcap, unsigned long long base) {
+  int i = threadIdx.x;
+  if (i < C_NUM * kCounterStride) ctrs[i] = 0;
+  __syncthreads();
+  if (i == 0) {
+    ctrs[C_QHEAD * kCounterStride] = base;
+    ctrs[C_QTAIL * kCounterStride] = base;
+    ctrs[C_QFREE * kCounterStride] = qcap;
+  }
+}
+
+__global__ void finalize_kernel(const unsigned long long* ctrs, unsigned long long* d_count) {
+  if (threadIdx.x == 0 && blockIdx.x == 0)
+    *d_count = ctrs[C_ERROR * kCounterStride] ? TDFS_COUNT_INVALID : ctrs[C_COUNT * kCounterStride];
+}
+
+using KernelFn = void (*)(const KParams);
+KernelFn pick_kernel(int mode, bool stats) {
+  if (mode == 0) return stats ? tdfs_kernel<0, true> : tdfs_kernel<0, false>;
+  return stats ? tdfs_kernel<1, true> : tdfs_kernel<1, false>;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+int cuda_fail(cudaError_t e, const char* what) {
+  return fail(TDFS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ host side
+int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int* out) {
+  (void)device;
+  int nb = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, pick_kernel(enumerate ? 1 : 0, stats), wpb * 32, 0);
+  if (e != cudaSuccess) return cuda_fail(e, "occupancy");
+  *out = std::max(1, nb);
+  return TDFS_OK;
+}
+
+int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayout* L) {
+  if (!g || !p || !o || !L) return fail(TDFS_E_INVALID_ARG, "layout: NULL");
+  if (o->chunk < 1 || o->chunk > 4096) return fail(TDFS_E_INVALID_ARG, "opts.chunk must be in [1, 4096]");
+  if (o->queue_ints < 3) return fail(TDFS_E_INVALID_ARG, "opts.queue_ints must be >= 3");
+  if (o->page_bytes < 128 || (o->page_bytes & (o->page_bytes - 1)))
+    return fail(TDFS_E_INVALID_ARG, "opts.page_bytes must be a power of two >= 128");
+  if (o->shard_world < 1 || o->shard_rank < 0 || o->shard_rank >= o->shard_world)
+    return fail(TDFS_E_INVALID_ARG, "opts.shard_rank/shard_world");
+  if (o->warps_per_block < 0 || o->blocks < 0 || o->page_table_entries < 0 || o->pool_bytes < 0)
+    return fail(TDFS_E_INVALID_ARG, "opts: negative size");
+  int dev = g->device;
+  int sms = 0;
+  cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) return cuda_fail(e, "device attribute");
+  L->wpb = o->warps_per_block > 0 ? o->warps_per_block : 4;
+  if (L->wpb > 32) return fail(TDFS_E_INVALID_ARG, "opts.warps_per_block must be <= 32");
+  if (o->blocks > 0) {
+    L->blocks = o->blocks;
+  } else {
+    int mn = INT_MAX;
+    for (int m = 0; m < 2; m++)
+      for (int s = 0; s < 2; s++) {
+        int nb = 0;
+        int rc = blocks_per_sm(dev, L->wpb, s != 0, m != 0, &nb);
+        if (rc) return rc;
+        mn = std::min(mn, nb);
+      }
+    L->blocks = sms * mn;
+  }
+  const long long n_warps = (long long)L->blocks * L->wpb;
+  L->n_levels = std::max(0, p->k - 3);
+  const int ints_per_page = o->page_bytes / 4;
+  int shift = 0;
+  while ((1 << shift) < ints_per_page) shift++;
+  L->page_shift = shift;
+  // a level holds at most min-operand-length <= d_max candidates
+  long long need = std::max<long long>(1, (g->dmax + ints_per_page - 1) / ints_per_page);
+  L->E = o->page_table_entries > 0 ? o->page_table_entries : (int)need;
+  L->qcap = (uint64_t)(o->queue_ints / 3);
+  if (o->pool_bytes > 0) {
+    L->n_pages = (uint64_t)(o->pool_bytes / o->page_bytes);
+  } else {
+    // one page per warp-level plus room for 256 warps to reach d_max on every level
+    L->n_pages = (uint64_t)n_warps * L->n_levels + (uint64_t)std::min<long long>(n_warps, 256) * L->n_levels * L->E;
+  }
+  if (L->n_levels == 0) L->n_pages = 0;
+  if (L->n_pages > 0xfffffff0ull) return fail(TDFS_E_INVALID_ARG, "pool too large for 32-bit page ids");
+  size_t off = 0;
+  L->ctr = off;
+  off += align_up(sizeof(unsigned long long) * C_NUM * kCounterStride, 256);
+  L->stats = off;
+  off += align_up(sizeof(unsigned long long) * S_NUM, 256);
+  L->slots = off;
+  off += align_up(sizeof(QSlot) * L->qcap, 256);
+  L->tables = off;
+  off += align_up(sizeof(uint32_t) * (size_t)n_warps * std::max(L->n_levels, 1) * L->E, 256);
+  L->pool = off;
+  off += align_up((size_t)L->n_pages * o->page_bytes, 256);
+  L->total = off;
+  return TDFS_OK;
+}
+
+int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
+               int mode, int32_t* d_out, uint64_t cap, uint64_t* d_count, bool sync, uint64_t* h_count,
+               tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap, int64_t* n_trace) {
+  WsLayout L;
+  int rc = resolve_layout(g, p, o, &L);
+  if (rc) return rc;
+  if (!ws || ((uintptr_t)ws & 255u)) return fail(TDFS_E_WORKSPACE, "workspace NULL or not 256-byte aligned");
+  if (ws_bytes < L.total) return fail(TDFS_E_WORKSPACE, "workspace smaller than tdfs_workspace_bytes()");
+  cudaError_t e = cudaSetDevice(g->device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice");
+  cudaStream_t st = (cudaStream_t)stream;
+  char* base = (char*)ws;
+  const bool want_stats = stats != nullptr;
+
+  KParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.offs = g->d_offs;
+  P.adj = g->d_adj;
+  P.src = g->d_src;
+  P.label = g->d_label;
+  P.n = g->n;
+  P.plan = p->dev;
+  P.shard_rank = o->shard_rank;
+  P.shard_world = o->shard_world;
+  P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
+  P.chunk = o->chunk;
+  P.n_levels = L.n_levels;
+  P.slots = (QSlot*)(base + L.slots);
+  P.qcap = L.qcap;
+  P.ctr = (unsigned long long*)(base + L.ctr);
+  P.stats = want_stats ? (unsigned long long*)(base + L.stats) : nullptr;
+  P.page_tables = (uint32_t*)(base + L.tables);
+  P.pool = (int32_t*)(base + L.pool);
+  P.n_pages = (uint32_t)L.n_pages;
+  P.page_shift = L.page_shift;
+  P.E = L.E;
+  P.tau_ns = o->tau_ns;
+  P.out = d_out;
+  P.cap = cap;
+  int32_t* d_trace = nullptr;
+  if (h_trace && trace_cap > 0) {
+    if ((e = cudaMalloc(&d_trace, sizeof(int32_t) * 3 * (size_t)trace_cap)) != cudaSuccess)
+      return fail(TDFS_E_OOM, "trace buffer");
+    P.trace = d_trace;
+    P.trace_cap = trace_cap;
+  }
+
+  const unsigned long long ticket_base = 0;
+  init_counters_kernel<<<1, C_NUM * kCounterStride, 0, st>>>(P.ctr, P.qcap, ticket_base);
+  if (want_stats) cudaMemsetAsync(P.stats, 0, sizeof(unsigned long long) * S_NUM, st);
+  {
+    int nb = (int)std::min<uint64_t>((L.qcap + 255) / 256, 4096);
+    init_queue_kernel<<<std::max(nb, 1), 256, 0, st>>>(P.slots, P.qcap, ticket_base);
+  }
+  size_t tbytes = sizeof(uint32_t) * (size_t)L.blocks * L.wpb * std::max(L.n_levels, 1) * L.E;
+  if (L.n_levels > 0) cudaMemsetAsync(P.page_tables, 0xff, tbytes, st);
+
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  if (want_stats) {
+    cudaEventCreate(&ev0);
+    cudaEventCreate(&ev1);
+    cudaEventRecord(ev0, st);
+  }
+  KernelFn fn = pick_kernel(mode, want_stats);
+  fn<<<L.blocks, L.wpb * 32, 0, st>>>(P);
+  if ((e = cudaGetLastError()) != cudaSuccess) {
+    cudaFree(d_trace);
+    return cuda_fail(e, "kernel launch");
+  }
+  if (want_stats) cudaEventRecord(ev1, st);
+  if (d_count) finalize_kernel<<<1, 32, 0, st>>>(P.ctr, (unsigned long long*)d_count);
+
+  if (!(sync || h_count || want_stats || h_trace)) return TDFS_OK;
+  unsigned long long hc[C_NUM * kCounterStride];
+  e = cudaMemcpyAsync(hc, P.ctr, sizeof(hc), cudaMemcpyDeviceToHost, st);
+  unsigned long long hs[S_NUM];
+  if (e == cudaSuccess && want_stats) e = cudaMemcpyAsync(hs, P.stats, sizeof(hs), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) {
+    cudaFree(d_trace);
+    return cuda_fail(e, "kernel execution");
+  }
+  if (h_trace && d_trace) {
+    long long nt = (long long)hc[C_TRACE * kCounterStride];
+    if (n_trace) *n_trace = nt;
+    long long ncp = std::min<long long>(nt, trace_cap);
+    if (ncp > 0) cudaMemcpy(h_trace, d_trace, sizeof(int32_t) * 3 * (size_t)ncp, cudaMemcpyDeviceToHost);
+    cudaFree(d_trace);
+  }
+  if (want_stats) {
+    std::memset(stats, 0, sizeof(*stats));
+    for (int i = 0; i < kMaxK + 1; i++) stats->nodes_per_level[i] = hs[S_NODES + i];
+    stats->adj_bytes = hs[S_ADJ_BYTES];
+    stats->tasks_enqueued = hs[S_ENQ];
+    stats->tasks_dequeued = hs[S_DEQ];
+    stats->timeouts = hs[S_TIMEOUTS];
+    stats->queue_full = hs[S_QFULL];
+    stats->edges_scanned = hs[S_EDGES_SCANNED];
+    stats->edges_filtered_in = hs[S_EDGES_IN];
+    stats->chunks_fetched = hs[S_CHUNKS];
+    stats->pages_used = std::min<unsigned long long>(hc[C_POOL * kCounterStride], L.n_pages);
+    stats->pool_pages = L.n_pages;
+    stats->grid_blocks = L.blocks;
+    stats->warps_per_block = L.wpb;
+    stats->page_table_entries = L.E;
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    stats->kernel_ms = ms;
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+  }
+  if (hc[C_ERROR * kCounterStride]) return fail(TDFS_E_STACK_EXHAUSTED, "stack page pool or page table exhausted "
+                                                "(raise pool_bytes / page_table_entries); no count produced");
+  if (h_count) *h_count = hc[C_COUNT * kCounterStride];
+  if (mode == 1 && cap < hc[C_COUNT * kCounterStride]) return TDFS_E_OUTPUT_OVERFLOW;
+  return TDFS_OK;
+}
+
+}  // namespace tdfs

@@ -102,6 +102,17 @@ def from_edge_list(n: int, pairs: Sequence[Tuple[int, int]], name: str = "custom
     return Graph(n, e, lab, name)
 
 
+def to_csr(g: Graph):
+    """Input-format conversion (symmetric CSR of a simple graph): offs int64[n+1], adj int32[2m]."""
+    a = np.concatenate([g.edges[:, 0], g.edges[:, 1]]).astype(np.int64)
+    b = np.concatenate([g.edges[:, 1], g.edges[:, 0]]).astype(np.int64)
+    idx = np.lexsort((b, a))
+    cnt = np.bincount(a, minlength=g.n)
+    offs = np.zeros(g.n + 1, np.int64)
+    np.cumsum(cnt, out=offs[1:])
+    return offs, np.ascontiguousarray(b[idx].astype(np.int32))
+
+
 def random_labels(n: int, num_labels: int, seed: int) -> np.ndarray:
     out = np.empty(n, dtype=np.uint8)
     _gen().tdfs_gen_labels(n, int(num_labels), int(seed), out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)))

@@ -1,0 +1,291 @@
+"""Parity of the CUDA path (through the C-ABI) with the CPU oracle, element by element.
+
+Counts and enumerated match sets are integer results: the bar is bit-exact equality.
+Sizes: small graphs the oracle finishes in seconds but which still span many warps,
+many 32-wide batches, ragged chunk tails, multi-page stack levels (tiny pages), and the
+timeout/queue path (tau = 0); then BASELINE.json's full-size configs on sampled shards
+(the oracle restricted to the same directed root edges) and closed forms at full size.
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle as O
+import tdfs_inputs as T
+from tests import golden_io as G
+from tests import gpu_util as U
+
+pytestmark = pytest.mark.gpu
+
+THREADS = max(1, min(64, os.cpu_count() or 1))
+
+ALL_Q = ["edge", "wedge", "triangle", "path3", "star3", "c4", "diamond", "tailed_triangle", "k4", "house", "c5",
+         "k5", "fig1_q", "prism", "w5", "c6", "k6", "k6_minus_e", "w6", "two_k4", "k7", "c8", "k8_minus_e"]
+
+
+# ------------------------------------------------------------------ Fig. 1
+def test_fig1_worked_example():
+    d = G.read("fig1.txt")
+    g = T.fig1_data()
+    q = T.query("fig1_q")
+    for cons, key in (([], "M_none"), ([(0, 2)], "M_u1_lt_u3"), ("auto", "M_auto")):
+        t, total, ovf = U.enumerate_sorted(g, q, cons if cons != [] else "none")
+        assert not ovf
+        assert sorted(tuple(int(x) + 1 for x in r) for r in t) == sorted(G.tuples(d[key]))
+    assert U.count(g, q, [(0, 2)]) == 2
+
+
+# ------------------------------------------------------------------ config 1
+@pytest.mark.parametrize("m", [10_000, 30_000])
+def test_config1_er_fig1_query(m):
+    g = T.erdos_renyi(2000, m, 1)
+    q = T.query("fig1_q")
+    for cons in ([(0, 2)], "auto", "none"):
+        assert U.count(g, q, cons) == O.count(g, q, cons), cons
+    t, total, _ = U.enumerate_sorted(g, q, [(0, 2)])
+    assert np.array_equal(t, O.enumerate_sorted(g, q, [(0, 2)]))
+
+
+def test_config1_planted():
+    g = T.plant(T.erdos_renyi(2000, 10_000, 1), T.fig1_data(), seed=5)
+    q = T.query("fig1_q")
+    ref = O.count(g, q, [(0, 2)])
+    assert ref >= 2
+    assert U.count(g, q, [(0, 2)]) == ref
+    assert U.count(g, q, "auto") == O.count(g, q, "auto")
+
+
+# --------------------------------------------------------- all queries, mid graphs
+@pytest.fixture(scope="module")
+def rmat12():
+    return T.rmat(12, 8, 3)
+
+
+@pytest.fixture(scope="module")
+def er_dense():
+    return T.erdos_renyi(400, 6000, 4)
+
+
+@pytest.mark.parametrize("name", ALL_Q)
+def test_counts_all_queries_rmat(rmat12, name):
+    q = T.query(name)
+    g = rmat12 if q.k <= 6 else T.rmat(10, 8, 3)
+    ref = O.count(g, q, "auto", threads=THREADS)
+    assert U.count(g, q, "auto") == ref
+    if q.k <= 5:
+        assert U.count(g, q, "none") == O.count(g, q, "none", threads=THREADS)
+
+
+@pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "k4", "house", "c5", "k5", "fig1_q", "prism", "w5"])
+def test_counts_dense_er(er_dense, name):
+    q = T.query(name)
+    assert U.count(er_dense, q, "auto") == O.count(er_dense, q, "auto", threads=THREADS)
+
+
+@pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "house", "fig1_q", "k5", "prism"])
+def test_enumerate_sets(rmat12, name):
+    q = T.query(name)
+    g = T.rmat(10, 8, 7)
+    t, total, ovf = U.enumerate_sorted(g, q, "auto")
+    ref = O.enumerate_sorted(g, q, "auto")
+    assert not ovf and total == ref.shape[0]
+    assert np.array_equal(t, ref)
+
+
+def test_enumerate_overflow_keeps_exact_total():
+    g = T.rmat(10, 8, 7)
+    q = T.query("triangle")
+    ref = O.count(g, q, "auto")
+    assert ref > 100
+    t, total, ovf = U.enumerate_sorted(g, q, "auto", cap=50)
+    assert ovf and total == ref and t.shape[0] == 50
+    E = set(map(tuple, g.edges.tolist()))
+    for r in t:
+        a, b, c = sorted(int(x) for x in r)
+        assert (a, b) in E and (a, c) in E and (b, c) in E
+
+
+# ------------------------------------------------------- settings must not change results
+@pytest.mark.parametrize("tau_ms", [None, 10.0, 0.0])
+@pytest.mark.parametrize("page_bytes", [8192, 128])
+def test_tau_and_page_invariance(rmat12, tau_ms, page_bytes):
+    for name in ["diamond", "house", "fig1_q", "c5", "prism"]:
+        q = T.query(name)
+        ref = O.count(rmat12, q, "auto", threads=THREADS)
+        got = U.count(rmat12, q, "auto", tau_ms=tau_ms, page_bytes=page_bytes)
+        assert got == ref, (name, tau_ms, page_bytes)
+
+
+def test_chunk_queue_grid_invariance(rmat12):
+    q = T.query("house")
+    ref = O.count(rmat12, q, "auto", threads=THREADS)
+    for kw in (dict(chunk=1), dict(chunk=32), dict(chunk=7, tau_ms=0.0, queue_ints=30),
+               dict(blocks=1, warps_per_block=1, tau_ms=0.0), dict(blocks=3, warps_per_block=2, tau_ms=0.0),
+               dict(tau_ms=0.0, queue_ints=3)):
+        assert U.count(rmat12, q, "auto", **kw) == ref, kw
+
+
+def test_order_independence(rmat12):
+    import random
+    rng = random.Random(3)
+    for name in ["diamond", "house", "fig1_q", "prism"]:
+        q = T.query(name)
+        ref = O.count(rmat12, q, "auto", threads=THREADS)
+        adj = {(a, b) for a, b in q.edges} | {(b, a) for a, b in q.edges}
+        for _ in range(3):
+            # random connected order
+            order = [rng.randrange(q.k)]
+            while len(order) < q.k:
+                cand = [u for u in range(q.k) if u not in order and any((u, w) in adj for w in order)]
+                order.append(rng.choice(cand))
+            assert U.count(rmat12, q, "auto", order=order) == ref, (name, order)
+
+
+def test_shard_sum(rmat12):
+    for name in ["triangle", "diamond", "house"]:
+        q = T.query(name)
+        ref = O.count(rmat12, q, "auto", threads=THREADS)
+        for W in (2, 3, 8):
+            assert sum(U.count(rmat12, q, "auto", shard_rank=r, shard_world=W) for r in range(W)) == ref
+
+
+def test_labeled_queries():
+    g = T.chung_lu(20_000, 120_000, 2.2, 600.0, 7).with_labels(8, 11)
+    for name in ["triangle", "c4", "house", "prism", "w5", "w6", "two_k4"]:
+        for nl in (8, 2):
+            q = T.labeled_query(name, nl)
+            assert U.count(g, q, "auto") == O.count(g, q, "auto", threads=THREADS), (name, nl)
+    # a single label equals unlabeled
+    g1 = T.Graph(g.n, g.edges, np.zeros(g.n, np.uint8), "one-label")
+    q = T.query("house")
+    assert U.count(g1, q.with_labels([0] * q.k), "auto") == O.count(g1, q, "auto", threads=THREADS)
+
+
+# ------------------------------------------------------------------ stats parity
+@pytest.mark.parametrize("name", ["triangle", "diamond", "house", "fig1_q", "prism"])
+def test_nodes_per_level_and_W_match_oracle(rmat12, name):
+    q = T.query(name)
+    order = O.oracle_order(q)
+    for tau in (None, 0.0):
+        cnt, st = U.count(rmat12, q, "auto", order=order, stats=True, tau_ms=tau)
+        r = O.match(rmat12, q, "auto", order=order, deg_filter=True, threads=THREADS)
+        assert cnt == r["count"]
+        assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k]
+        assert st["adj_bytes"] == r["W"]
+
+
+def test_stack_exhaustion_is_an_error_never_a_count():
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    g = T.rmat(12, 8, 3)
+    q = T.query("house")
+    with pytest.raises(M.TdfsError) as e:
+        U.count(g, q, "auto", page_bytes=128, pool_bytes=128 * 4)
+    assert e.value.status == M.TDFS_E_STACK_EXHAUSTED
+    with pytest.raises(M.TdfsError) as e:
+        U.count(g, q, "auto", page_bytes=128, page_table_entries=1)
+    assert e.value.status == M.TDFS_E_STACK_EXHAUSTED
+
+
+# ------------------------------------------------------------------ edge cases
+def test_edge_cases():
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    empty = T.Graph(10, np.zeros((0, 2), np.int32), None, "empty")
+    assert U.count(empty, T.query("triangle"), "auto") == 0
+    one = T.from_edge_list(3, [(0, 1)])
+    assert U.count(one, T.query("edge"), "auto") == 1
+    assert U.count(one, T.query("edge"), "none") == 2
+    assert U.count(one, T.query("triangle"), "auto") == 0
+    K = T.complete(9)
+    for k in range(3, 9):
+        assert U.count(K, T.query("triangle" if k == 3 else f"k{k}"), "auto") == math.comb(9, k)
+    assert U.count(K, T.query("c4"), "none") == math.perm(9, 4)
+    # labels that do not occur
+    g = T.rmat(8, 8, 1).with_labels(2, 3)
+    q = T.query("triangle").with_labels([5, 5, 5])
+    assert U.count(g, q, "auto") == 0
+    # contradictory constraints give 0, never an error
+    assert U.count(K, T.query("triangle"), [(0, 1), (1, 0)]) == 0
+    # duplicate / reversed / self-loop edges in the input are normalised
+    h = M.tdfs_load_edges(4, np.array([[0, 1], [1, 0], [1, 2], [2, 2], [2, 0], [0, 1]]))
+    p = M.plan_from_query(T.query("triangle"))
+    assert M.tdfs_count(h, p) == 1
+    assert h.info()["m"] == 3
+
+
+def test_invalid_csr_rejected():
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    offs = np.array([0, 2, 3, 4], np.int64)
+    adj = np.array([2, 1, 0, 0], np.int32)  # unsorted list of vertex 0
+    with pytest.raises(M.TdfsError) as e:
+        M.tdfs_load_graph(offs, adj, validate=True)
+    assert e.value.status == M.TDFS_E_GRAPH_FORMAT
+    h = M.tdfs_load_graph(offs, adj, normalize=True)
+    assert h.info()["m"] == 2
+    bad = np.array([0, 1, 2, 2], np.int64)
+    with pytest.raises(M.TdfsError) as e:
+        M.tdfs_load_graph(bad, np.array([7, 0], np.int32), validate=True)
+    assert e.value.status in (M.TDFS_E_GRAPH_FORMAT, M.TDFS_E_ID_RANGE)
+
+
+def _numpy_csr(g):
+    """Input-format conversion for the DEVICE_BORROW test (plain numpy, no matching)."""
+    a = np.concatenate([g.edges[:, 0], g.edges[:, 1]]).astype(np.int64)
+    b = np.concatenate([g.edges[:, 1], g.edges[:, 0]]).astype(np.int64)
+    idx = np.lexsort((b, a))
+    offs = np.zeros(g.n + 1, np.int64)
+    np.add.at(offs, a + 1, 1)
+    return np.cumsum(offs), b[idx].astype(np.int32)
+
+
+def test_device_borrow_csr():
+    import torch
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    g = T.rmat(10, 8, 9)
+    offs, adj = _numpy_csr(g)
+    to = torch.from_numpy(offs).cuda()
+    ta = torch.from_numpy(adj).cuda()
+    hb = M.tdfs_load_graph(to, ta, validate=True)
+    assert hb.info()["m"] == g.m
+    p = M.plan_from_query(T.query("diamond"))
+    assert M.tdfs_count(hb, p) == O.count(g, T.query("diamond"), "auto")
+    bad = ta.clone()
+    bad[0], bad[1] = ta[1], ta[0]  # break the order of the first list
+    with pytest.raises(M.TdfsError):
+        M.tdfs_load_graph(to, bad, validate=True)
+
+
+# ------------------------------------------------------------------ full-size configs
+@pytest.fixture(scope="module")
+def c2():
+    return T.config_graph(2)
+
+
+def test_config2_full_triangle_and_closed_forms(c2):
+    q = T.query("triangle")
+    assert U.count(c2, q, "auto") == O.count(c2, q, "auto", threads=THREADS)
+    d = np.bincount(c2.edges.reshape(-1), minlength=c2.n).astype(object)
+    assert U.count(c2, T.query("wedge"), "auto") == int(sum(x * (x - 1) // 2 for x in d))
+    assert U.count(c2, T.query("star3"), "auto") == int(sum(x * (x - 1) * (x - 2) // 6 for x in d))
+
+
+@pytest.mark.parametrize("name", ["c4", "diamond", "tailed_triangle", "k4"])
+def test_config2_full_sampled_shards(c2, name):
+    """Full C2 graph in the bench launch configuration; the oracle computes the matches
+    rooted at the sampled shard's directed edges (same order, so the same root edges)."""
+    q = T.query(name)
+    order = O.oracle_order(q)
+    W = 4001
+    for r in (0, 1777):
+        got = U.count(c2, q, "auto", order=order, shard_rank=r, shard_world=W)
+        ref = O.count(c2, q, "auto", order=order, shard=(r, W), threads=THREADS)
+        assert got == ref, (name, r)
+
+
+def test_config2_auto_order_full_counts_equal_explicit_order(c2):
+    """The planner's own order (what bench.py runs) gives the same full count as the
+    oracle-order run whose shards are checked above."""
+    for name in ["c4", "diamond", "tailed_triangle", "k4"]:
+        q = T.query(name)
+        assert U.count(c2, q, "auto") == U.count(c2, q, "auto", order=O.oracle_order(q))
