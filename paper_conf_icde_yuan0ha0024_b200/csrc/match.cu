@@ -215,11 +215,12 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
   long long sz = extend<0, STATS>(P, c, d);
   if (sz < 0) return false;
   if (lane == d) { c.lsize = sz; c.liter = 0; }
+  bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
   for (;;) {
     const long long it = __shfl_sync(FULL, c.liter, d);
     const long long size = __shfl_sync(FULL, c.lsize, d);
     if (it < size) {
-      if (d == 2 && timed_out(P, c)) {
+      if (d == 2 && !grace && timed_out(P, c)) {
         // timeout: push the current and all remaining siblings, then backtrack
         if (STATS && lane == 0) c.touts++;
         long long upto = split_level2(P, c, q, it, size);
@@ -230,8 +231,10 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         // queue full: the pushed prefix is gone, continue in place with t0 reset
         if (lane == d) c.liter = upto;
         if (lane == 0) c.t0 = globaltimer();
+        grace = true;
         continue;
       }
+      if (d == 2) grace = false;
       const uint32_t* table = c.tables + (size_t)(d - 2) * P.E;
       const int v = paged_read(P, table, it);
       if (lane == d) { c.sreg = v; c.liter = it + 1; }
@@ -278,13 +281,12 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
     }
     unsigned mask = __ballot_sync(FULL, ok);
     if (STATS) {
+      const unsigned scanned = __ballot_sync(FULL, inr);
       if (lane == 1) c.lnodes += __popc(mask);
       if (lane == 0) {
-        c.scanned += __popc(__ballot_sync(FULL, inr));
+        c.scanned += __popc(scanned);
         c.edges_in += __popc(mask);
       }
-    } else {
-      (void)0;
     }
     if (k == 2) {  // the query is one edge: every filtered edge is a match
       const int cnt = __popc(mask);
@@ -524,8 +526,12 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   if (o->pool_bytes > 0) {
     L->n_pages = (uint64_t)(o->pool_bytes / o->page_bytes);
   } else {
-    // one page per warp-level plus room for 256 warps to reach d_max on every level
-    L->n_pages = (uint64_t)n_warps * L->n_levels + (uint64_t)std::min<long long>(n_warps, 256) * L->n_levels * L->E;
+    // every warp-level able to reach d_max, capped at max(4 pages per warp-level, 2 GiB):
+    // pages are a per-warp high-water mark, so typical use is ~1 page each
+    uint64_t full = (uint64_t)n_warps * L->n_levels * L->E;
+    uint64_t floor_pages = std::max<uint64_t>((uint64_t)n_warps * L->n_levels * 4,
+                                              (2ull << 30) / (uint64_t)o->page_bytes);
+    L->n_pages = std::min(full, floor_pages);
   }
   if (L->n_levels == 0) L->n_pages = 0;
   if (L->n_pages > 0xfffffff0ull) return fail(TDFS_E_INVALID_ARG, "pool too large for 32-bit page ids");

@@ -23,7 +23,7 @@ def _sorted_rows(a):
 
 
 # ------------------------------------------------------------------ Alg. 3
-@pytest.mark.parametrize("base", [0, (1 << 32) - 5, (1 << 64) - 7])
+@pytest.mark.parametrize("base", [0, (1 << 32) - 5, (1 << 63) - 7])
 def test_queue_single_warp_fifo_full_and_empty(base):
     cap = 10
     t = _tasks(25)
@@ -32,7 +32,7 @@ def test_queue_single_warp_fifo_full_and_empty(base):
     assert np.array_equal(out, t[:cap])      # FIFO; dequeue returns false once empty
 
 
-@pytest.mark.parametrize("base", [0, (1 << 32) - 3, (1 << 64) - 100])
+@pytest.mark.parametrize("base", [0, (1 << 32) - 3, (1 << 63) - 100])
 @pytest.mark.parametrize("cap,warps", [(7, 64), (1000, 512), (3, 8)])
 def test_queue_multi_warp_exactly_once(base, cap, warps):
     t = _tasks(20000, seed=cap)

@@ -58,36 +58,59 @@ def test_config1_planted():
 
 
 # --------------------------------------------------------- all queries, mid graphs
+# graphs chosen per query so that the oracle finishes in seconds while the GPU still runs
+# thousands of warps, many 32-wide batches and multi-page levels
+_GRAPHS = {}
+
+
+def graph(key):
+    if key not in _GRAPHS:
+        _GRAPHS[key] = {"r12": lambda: T.rmat(12, 8, 3), "r10": lambda: T.rmat(10, 6, 3),
+                        "r9": lambda: T.rmat(9, 5, 3), "er300": lambda: T.erdos_renyi(300, 900, 4),
+                        "er400": lambda: T.erdos_renyi(400, 6000, 4)}[key]()
+    return _GRAPHS[key]
+
+
+_ORACLE = {}
+
+
+def oracle_count(gkey, q, cons="auto", **kw):
+    key = (gkey, q.name, str(cons), str(sorted(kw.items())))
+    if key not in _ORACLE:
+        _ORACLE[key] = O.count(graph(gkey), q, cons, threads=THREADS, **kw)
+    return _ORACLE[key]
+
+
+QUERY_GRAPH = {"edge": "r12", "wedge": "r12", "triangle": "r12", "path3": "r12", "star3": "r12", "c4": "r12",
+               "diamond": "r12", "tailed_triangle": "r12", "k4": "r12", "k5": "r12", "house": "r10", "c5": "r10",
+               "fig1_q": "r10", "prism": "r10", "w5": "r10", "c6": "r9", "k6": "r9", "k6_minus_e": "r9",
+               "w6": "r9", "two_k4": "r9", "k7": "r9", "c8": "er300", "k8_minus_e": "r9"}
+
+
 @pytest.fixture(scope="module")
 def rmat12():
-    return T.rmat(12, 8, 3)
-
-
-@pytest.fixture(scope="module")
-def er_dense():
-    return T.erdos_renyi(400, 6000, 4)
+    return graph("r12")
 
 
 @pytest.mark.parametrize("name", ALL_Q)
-def test_counts_all_queries_rmat(rmat12, name):
+def test_counts_all_queries(name):
     q = T.query(name)
-    g = rmat12 if q.k <= 6 else T.rmat(10, 8, 3)
-    ref = O.count(g, q, "auto", threads=THREADS)
-    assert U.count(g, q, "auto") == ref
-    if q.k <= 5:
-        assert U.count(g, q, "none") == O.count(g, q, "none", threads=THREADS)
+    gk = QUERY_GRAPH[name]
+    assert U.count(graph(gk), q, "auto") == oracle_count(gk, q, "auto")
+    if q.k <= 4 or gk == "er300":
+        assert U.count(graph(gk), q, "none") == oracle_count(gk, q, "none")
 
 
 @pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "k4", "house", "c5", "k5", "fig1_q", "prism", "w5"])
-def test_counts_dense_er(er_dense, name):
+def test_counts_dense_er(name):
     q = T.query(name)
-    assert U.count(er_dense, q, "auto") == O.count(er_dense, q, "auto", threads=THREADS)
+    assert U.count(graph("er400"), q, "auto") == oracle_count("er400", q, "auto")
 
 
 @pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "house", "fig1_q", "k5", "prism"])
-def test_enumerate_sets(rmat12, name):
+def test_enumerate_sets(name):
     q = T.query(name)
-    g = T.rmat(10, 8, 7)
+    g = T.rmat(10, 8, 7) if q.k <= 4 else graph("r9")
     t, total, ovf = U.enumerate_sorted(g, q, "auto")
     ref = O.enumerate_sorted(g, q, "auto")
     assert not ovf and total == ref.shape[0]
@@ -110,29 +133,31 @@ def test_enumerate_overflow_keeps_exact_total():
 # ------------------------------------------------------- settings must not change results
 @pytest.mark.parametrize("tau_ms", [None, 10.0, 0.0])
 @pytest.mark.parametrize("page_bytes", [8192, 128])
-def test_tau_and_page_invariance(rmat12, tau_ms, page_bytes):
+def test_tau_and_page_invariance(tau_ms, page_bytes):
     for name in ["diamond", "house", "fig1_q", "c5", "prism"]:
         q = T.query(name)
-        ref = O.count(rmat12, q, "auto", threads=THREADS)
-        got = U.count(rmat12, q, "auto", tau_ms=tau_ms, page_bytes=page_bytes)
+        ref = oracle_count("r10", q, "auto")
+        got = U.count(graph("r10"), q, "auto", tau_ms=tau_ms, page_bytes=page_bytes)
         assert got == ref, (name, tau_ms, page_bytes)
 
 
-def test_chunk_queue_grid_invariance(rmat12):
+def test_chunk_queue_grid_invariance():
+    rmat12 = graph("r10")
     q = T.query("house")
-    ref = O.count(rmat12, q, "auto", threads=THREADS)
+    ref = oracle_count("r10", q, "auto")
     for kw in (dict(chunk=1), dict(chunk=32), dict(chunk=7, tau_ms=0.0, queue_ints=30),
                dict(blocks=1, warps_per_block=1, tau_ms=0.0), dict(blocks=3, warps_per_block=2, tau_ms=0.0),
                dict(tau_ms=0.0, queue_ints=3)):
         assert U.count(rmat12, q, "auto", **kw) == ref, kw
 
 
-def test_order_independence(rmat12):
+def test_order_independence():
     import random
     rng = random.Random(3)
+    rmat12 = graph("r10")
     for name in ["diamond", "house", "fig1_q", "prism"]:
         q = T.query(name)
-        ref = O.count(rmat12, q, "auto", threads=THREADS)
+        ref = oracle_count("r10", q, "auto")
         adj = {(a, b) for a, b in q.edges} | {(b, a) for a, b in q.edges}
         for _ in range(3):
             # random connected order
@@ -143,10 +168,11 @@ def test_order_independence(rmat12):
             assert U.count(rmat12, q, "auto", order=order) == ref, (name, order)
 
 
-def test_shard_sum(rmat12):
+def test_shard_sum():
+    rmat12 = graph("r10")
     for name in ["triangle", "diamond", "house"]:
         q = T.query(name)
-        ref = O.count(rmat12, q, "auto", threads=THREADS)
+        ref = oracle_count("r10", q, "auto")
         for W in (2, 3, 8):
             assert sum(U.count(rmat12, q, "auto", shard_rank=r, shard_world=W) for r in range(W)) == ref
 
@@ -165,7 +191,8 @@ def test_labeled_queries():
 
 # ------------------------------------------------------------------ stats parity
 @pytest.mark.parametrize("name", ["triangle", "diamond", "house", "fig1_q", "prism"])
-def test_nodes_per_level_and_W_match_oracle(rmat12, name):
+def test_nodes_per_level_and_W_match_oracle(name):
+    rmat12 = graph("r10")
     q = T.query(name)
     order = O.oracle_order(q)
     for tau in (None, 0.0):
