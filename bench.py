@@ -45,6 +45,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--queries", type=str, default="")
     ap.add_argument("--cpu-sample-world", type=int, default=2001)
+    ap.add_argument("--profile-shard-world", type=int, default=1,
+                    help="profiling only: run shard 0 of W on one GPU (not a bench number)")
+    ap.add_argument("--flags", type=int, default=0, help="tdfs_run_opts.flags (ablations)")
     return ap.parse_args()
 
 
@@ -211,7 +214,7 @@ def run_ours(a):
     plans = [M.plan_from_query(q) for q in qs]
     plan_s = time.perf_counter() - t_plan0
     tau = None if a.tau_ms < 0 else a.tau_ms
-    opts = M.default_opts(tau_ms=tau, shard_rank=rank, shard_world=world)
+    opts = M.default_opts(tau_ms=tau, shard_rank=rank, shard_world=world * a.profile_shard_world, flags=a.flags)
     ws_bytes = max(M.tdfs_workspace_bytes(h, p, opts) for p in plans)
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
     d_counts = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")

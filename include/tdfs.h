@@ -141,6 +141,9 @@ void tdfs_free_plan(tdfs_plan* p);
  */
 #define TDFS_RUN_STATS 1u           /* fill tdfs_stats (slower kernel variant) */
 #define TDFS_RUN_TRACE 2u           /* test hook: record enqueued tasks (see tdfs_test.h) */
+#define TDFS_RUN_NO_REUSE 4u        /* ablation: disable set-intersection result reuse */
+#define TDFS_RUN_NO_SHORTCUT 8u     /* ablation: always scan the last level (no count-only window shortcut) */
+#define TDFS_RUN_NO_HUB_BITMAP 16u  /* ablation: probe hub adjacency lists by search, not by bitmap */
 
 typedef struct {
   int64_t tau_ns;              /* timeout tau; default 10 ms;

@@ -18,7 +18,7 @@ from typing import Optional, Sequence, Tuple, Union
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libtdfs.so")
+LIB_PATH = os.environ.get("TDFS_LIB") or os.path.join(_PKG, "libtdfs.so")  # TDFS_LIB: experiment variants
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libtdfs.so not found at {LIB_PATH}: build it first "
@@ -41,6 +41,9 @@ TDFS_GRAPH_VALIDATE = 1
 TDFS_GRAPH_NORMALIZE = 2
 TDFS_RUN_STATS = 1
 TDFS_RUN_TRACE = 2
+TDFS_RUN_NO_REUSE = 4
+TDFS_RUN_NO_SHORTCUT = 8
+TDFS_RUN_NO_HUB_BITMAP = 16
 TDFS_COUNT_INVALID = (1 << 64) - 1
 
 

@@ -34,9 +34,9 @@ def nvcc() -> str:
     raise RuntimeError("nvcc not found")
 
 
-def _compile(src: str, verbose_ptxas: bool) -> str:
-    obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-    cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-I", INCLUDE, "-I", CSRC,
+def _compile(src: str, verbose_ptxas: bool, defines=(), build_dir=None) -> str:
+    obj = os.path.join(build_dir or BUILD, os.path.basename(src) + ".o")
+    cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-I", INCLUDE, "-I", CSRC, *[f"-D{d}" for d in defines],
            "-Xcompiler", "-fPIC,-O3,-Wall", "--expt-relaxed-constexpr", "-c", os.path.join(CSRC, src), "-o", obj]
     if src.endswith(".cpp"):
         cmd[cmd.index("-c"):cmd.index("-c")] = ["-x", "cu"]
@@ -59,19 +59,22 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose_ptxas: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose_ptxas: bool = False, defines=(), out=None) -> str:
+    """Build libtdfs.so (or, for experiments, a variant with extra -D defines at `out`)."""
+    target = out or OUT
+    if not force and out is None and not _stale():
         return OUT
-    os.makedirs(BUILD, exist_ok=True)
+    bdir = BUILD if out is None else BUILD + "_" + os.path.basename(out).replace(".so", "")
+    os.makedirs(bdir, exist_ok=True)
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
-        objs = list(ex.map(lambda s: _compile(s, verbose_ptxas), SOURCES))
-    tmp = OUT + f".tmp{os.getpid()}"
+        objs = list(ex.map(lambda s: _compile(s, verbose_ptxas, defines, bdir), SOURCES))
+    tmp = target + f".tmp{os.getpid()}"
     cmd = [nvcc(), *ARCH, "-shared", "-o", tmp, *objs, "-Xcompiler", "-fPIC", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, OUT)
-    return OUT
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
 #include <cstring>
 #include <thread>
 
@@ -156,6 +157,71 @@ __global__ void scan_graph_kernel(const int64_t* __restrict__ offs, const int32_
   if (lmax) atomicMax(&out[2], lmax);
 }
 
+__global__ void hub_bits_kernel(const int64_t* __restrict__ offs, const int32_t* __restrict__ adj,
+                                const int32_t* __restrict__ hub_vertex, long long n_hubs, long long words,
+                                uint32_t* __restrict__ bits) {
+  for (long long h = blockIdx.x; h < n_hubs; h += gridDim.x) {
+    const int32_t v = hub_vertex[h];
+    uint32_t* row = bits + h * words;
+    for (long long e = offs[v] + threadIdx.x; e < offs[v + 1]; e += blockDim.x) {
+      const int32_t w = adj[e];
+      atomicOr(row + (w >> 5), 1u << (w & 31));
+    }
+  }
+}
+
+// Hub adjacency bitmaps: the highest-degree vertices (degree >= 256,
+// at most `budget` bytes of bitmaps) get an n-bit membership bitmap so that probing
+// w in N(hub) during Eq. (1) is one load instead of a binary search over a long list.
+int build_hub_bitmaps(Graph& G, cudaStream_t st) {
+  const long long words = (G.n + 31) / 32;
+  if (G.n == 0 || words == 0) return TDFS_OK;
+  long long budget = 64ll << 20;
+  if (const char* e = getenv("TDFS_HUB_BUDGET_MB")) budget = atoll(e) << 20;
+  const long long max_hubs = budget / (words * 4);
+  if (max_hubs <= 0) return TDFS_OK;
+  std::vector<int64_t> offs((size_t)G.n + 1);
+  cudaError_t e = cudaMemcpyAsync(offs.data(), G.d_offs, sizeof(int64_t) * (G.n + 1), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(e, "hubs: offs copy");
+  std::vector<std::pair<int64_t, int32_t>> cand;
+  const int64_t min_deg = 256;
+  for (int64_t v = 0; v < G.n; v++) {
+    int64_t d = offs[v + 1] - offs[v];
+    if (d >= min_deg) cand.push_back({-d, (int32_t)v});
+  }
+  if (cand.empty()) return TDFS_OK;
+  if ((long long)cand.size() > max_hubs) {
+    std::nth_element(cand.begin(), cand.begin() + max_hubs, cand.end());
+    cand.resize(max_hubs);
+  }
+  std::sort(cand.begin(), cand.end());
+  std::vector<int32_t> hub_id((size_t)G.n, -1), hub_vertex(cand.size());
+  for (size_t h = 0; h < cand.size(); h++) {
+    hub_vertex[h] = cand[h].second;
+    hub_id[cand[h].second] = (int32_t)h;
+  }
+  G.n_hubs = (int64_t)cand.size();
+  G.hub_words = words;
+  G.hub_min_deg = -cand.back().first;
+  int32_t* d_vert = nullptr;
+  if ((e = cudaMalloc(&G.d_hub_id, sizeof(int32_t) * G.n)) != cudaSuccess ||
+      (e = cudaMalloc(&G.d_hub_bits, sizeof(uint32_t) * (size_t)(G.n_hubs * words))) != cudaSuccess ||
+      (e = cudaMalloc(&d_vert, sizeof(int32_t) * G.n_hubs)) != cudaSuccess) {
+    cudaFree(d_vert);
+    return fail(TDFS_E_OOM, "hubs: alloc");
+  }
+  cudaMemcpyAsync(G.d_hub_id, hub_id.data(), sizeof(int32_t) * G.n, cudaMemcpyHostToDevice, st);
+  cudaMemcpyAsync(d_vert, hub_vertex.data(), sizeof(int32_t) * G.n_hubs, cudaMemcpyHostToDevice, st);
+  cudaMemsetAsync(G.d_hub_bits, 0, sizeof(uint32_t) * (size_t)(G.n_hubs * words), st);
+  hub_bits_kernel<<<(int)std::min<int64_t>(G.n_hubs, 65535), 256, 0, st>>>(G.d_offs, G.d_adj, d_vert, G.n_hubs, words,
+                                                                         G.d_hub_bits);
+  e = cudaStreamSynchronize(st);
+  cudaFree(d_vert);
+  if (e != cudaSuccess) return cuda_fail(e, "hubs: build");
+  return TDFS_OK;
+}
+
 int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enforce = false) {
   cudaError_t e;
   if ((e = cudaMalloc(&G.d_src, sizeof(int32_t) * (size_t)std::max<int64_t>(G.nnz, 1))) != cudaSuccess)
@@ -180,7 +246,7 @@ int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enf
     G.nlabels = G.d_label ? (int32_t)h[2] + 1 : 1;
   }
   if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "load: sync");
-  return TDFS_OK;
+  return build_hub_bitmaps(G, st);
 }
 
 void release(Graph& G) {
@@ -190,7 +256,10 @@ void release(Graph& G) {
     cudaFree(G.d_label);
   }
   cudaFree(G.d_src);
+  cudaFree(G.d_hub_id);
+  cudaFree(G.d_hub_bits);
   G.d_offs = nullptr; G.d_adj = nullptr; G.d_label = nullptr; G.d_src = nullptr;
+  G.d_hub_id = nullptr; G.d_hub_bits = nullptr; G.n_hubs = 0;
 }
 
 int upload(Graph& G, const int64_t* offs, const int32_t* adj, const uint8_t* label, cudaStream_t st) {

@@ -30,7 +30,9 @@ struct DevPlan {
   int32_t label[kMaxK];      // required label, -1 = any
   int32_t deg_min[kMaxK];    // degree filter threshold (0 = off), R8
   int32_t edge_cons;         // constraint between positions 0 and 1: +1 S0<S1, -1 S1<S0, 0 none
-  int32_t pad_;
+  int32_t reuse_enabled;     // set-intersection result reuse on
+  int8_t reuse[kMaxK];       // stored position r whose candidate list C(r) is a superset start for p, -1 none
+  uint8_t shortcut[kMaxK];   // last position: count without scanning; bit0 valid with reuse, bit1 without
 };
 
 struct Plan {
@@ -53,6 +55,10 @@ struct Graph {
   uint8_t* d_label = nullptr;
   int32_t* d_src = nullptr;  // source vertex of each directed entry (edge tasks)
   bool owns_csr = true;
+  // hub adjacency bitmaps: membership w in N(h) in O(1) for the highest-degree vertices
+  int32_t* d_hub_id = nullptr;     // [n], -1 for non-hubs
+  uint32_t* d_hub_bits = nullptr;  // [n_hubs][hub_words]
+  int64_t n_hubs = 0, hub_words = 0, hub_min_deg = 0;
 };
 
 // ---------------------------------------------------------------- device job
@@ -100,6 +106,12 @@ struct KParams {
   int32_t page_shift;          // log2(ints per page)
   int32_t E;                   // page-table entries per level
   int64_t tau_ns;              // < 0: infinity
+  int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
+  int32_t bsearch_variant;     // 0 halving, 1 power-of-two (experiments)
+  // hub bitmaps (nullptr when off)
+  const int32_t* hub_id;
+  const uint32_t* hub_bits;
+  long long hub_words;
   // enumerate
   int32_t* out;
   unsigned long long cap;

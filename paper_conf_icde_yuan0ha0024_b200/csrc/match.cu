@@ -33,6 +33,7 @@
 
 #include <algorithm>
 #include <climits>
+#include <cstdlib>
 #include <cstring>
 
 #include "internal.h"
@@ -47,7 +48,7 @@ template <bool STATS>
 struct Ctx {
   int lane;
   int sreg;                 // lane p: S[p]
-  long long lsize, liter;   // lane p: size[p], iter[p]
+  int lsize, liter;         // lane p: size[p], iter[p] (a level holds <= d_max < 2^31 ids)
   unsigned long long count;  // warp-uniform
   unsigned long long t0;     // lane 0: task start time
   unsigned long long lnodes; // lane p: nodes[p]   (STATS)
@@ -66,58 +67,125 @@ __device__ __forceinline__ bool timed_out(const KParams& P, Ctx<STATS>& c) {
   return __shfl_sync(FULL, t, 0) != 0;
 }
 
+// lower_bound of v in the paged list [lo, hi) of a stored level
+__device__ __forceinline__ long long paged_lower_bound(const KParams& P, const uint32_t* table, long long lo,
+                                                       long long hi, int v) {
+  while (lo < hi) {
+    long long mid = (lo + hi) >> 1;
+    if (paged_read(P, table, mid) < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
 // Candidate generation for position d (Eq. 1 + fused filters).
 // MODE_OUT: 0 = store into the paged level of d; 1 = count only (last position);
 //           2 = enumerate (last position).
+// allow_reuse2: the stored list of position 2 belongs to this prefix (false for tasks
+// <v1,v2,v3> taken from Q_task, whose level 2 was built by another warp).
 // Returns the number of candidates, or -1 on stack exhaustion.
 template <int MODE_OUT, bool STATS>
-__device__ long long extend(const KParams& P, Ctx<STATS>& c, int d) {
+__device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_reuse2) {
   const int lane = c.lane;
   const DevPlan& pl = P.plan;
-  const uint32_t bm = pl.bwd[d];
+  int r = pl.reuse[d];
+  if (r == 2 && !allow_reuse2) r = -1;
+  const uint32_t bm_all = pl.bwd[d];
+  // set-intersection result reuse: start from C(r), intersect the rest
+  const uint32_t bm = (r >= 0) ? (bm_all & ~pl.bwd[r]) : bm_all;
   const int nops = __popc(bm);
-  // operand t (lane t < nops) = adjacency list of S[j_t], j_t = t-th set bit of bm
+  // global operand t (lane t < nops) = adjacency list of S[j_t], j_t = t-th set bit of bm
   int jt = 0;
   {
     uint32_t m = bm;
     for (int i = 0; i < lane && m; i++) m &= m - 1;
     jt = m ? (__ffs(m) - 1) : 0;
   }
-  int sj = __shfl_sync(FULL, c.sreg, jt);
+  const int sj = __shfl_sync(FULL, c.sreg, jt);
   long long ob = 0, oe = 0;
+  int hid = -1;
   if (lane < nops) {
     ob = __ldg(P.offs + sj);
     oe = __ldg(P.offs + sj + 1);
+    if (P.hub_id) hid = __ldg(P.hub_id + sj);
   }
-  if (STATS) {
-    unsigned long long wb = (lane < nops) ? (unsigned long long)(4 * (oe - ob) + 16) : 0ull;
+  if (STATS) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
+    const bool mine = (bm_all >> lane) & 1u;
+    unsigned long long wb = 0;
+    if (mine) wb = (unsigned long long)(4 * (__ldg(P.offs + c.sreg + 1) - __ldg(P.offs + c.sreg)) + 16);
     for (int o = 16; o > 0; o >>= 1) wb += __shfl_xor_sync(FULL, wb, o);
     if (lane == 0) c.wbytes += wb;
   }
   // constraint window [lo, hi)
   const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
-  int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
-  int hi = __reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
+  const int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
+  const int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
   if (lo >= hi) return 0;
-  if (lane < nops && (lo > 0 || hi < INT_MAX)) {
+  const bool windowed = (lo > 0 || hi < INT_MAX);
+  if (lane < nops && windowed) {
     const int32_t* L = P.adj + ob;
-    int n = (int)(oe - ob);
-    int a = lo > 0 ? lower_bound_dev(L, n, lo) : 0;
-    int b = hi < INT_MAX ? a + lower_bound_dev(L + a, n - a, hi) : n;
+    const int n = (int)(oe - ob);
+    const int a = lo > 0 ? lower_bound_dev(L, n, lo) : 0;
+    const int b = hi < INT_MAX ? a + lower_bound_dev(L + a, n - a, hi) : n;
     oe = ob + b;
     ob = ob + a;
   }
-  long long len = (lane < nops) ? (oe - ob) : LLONG_MAX;
-  // shortest operand
-  unsigned minlen = __reduce_min_sync(FULL, (unsigned)min(len, (long long)UINT_MAX));
-  if (minlen == 0) return 0;
-  int tA = __ffs(__ballot_sync(FULL, lane < nops && (unsigned)len == minlen)) - 1;
-  const long long bA = __shfl_sync(FULL, ob, tA);
-  const long long eA = __shfl_sync(FULL, oe, tA);
-  const uint32_t others = __ballot_sync(FULL, lane < nops && lane != tA);
+  // the reused list, windowed
+  const uint32_t* rtable = nullptr;
+  long long ra = 0, rb = 0;
+  if (r >= 0) {
+    rtable = c.tables + (size_t)(r - 2) * P.E;
+    const long long rsize = __shfl_sync(FULL, c.lsize, r);
+    ra = lo > 0 ? paged_lower_bound(P, rtable, 0, rsize, lo) : 0;
+    rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
+    if (ra >= rb) return 0;
+  }
   const uint32_t injm = pl.inj_mask[d];
-  const int need_label = pl.label[d];
-  const int dmin = pl.deg_min[d];
+
+  // count-only last position with a single remaining list and no per-element filter:
+  // |C(d)| = |window| - |matched vertices inside it| (no scan)
+  if (MODE_OUT == 1 && (pl.shortcut[d] & (r >= 0 ? 1u : 2u)) && (r >= 0 || nops == 1)) {
+    const long long b0 = __shfl_sync(FULL, ob, 0), e0 = __shfl_sync(FULL, oe, 0);
+    const long long len = (r >= 0) ? (rb - ra) : (e0 - b0);
+    bool hit = false;
+    if ((injm >> lane) & 1u) {
+      const int s = c.sreg;
+      if (s >= lo && s < hi && len > 0) {
+        if (r >= 0) {
+          const long long i = paged_lower_bound(P, rtable, ra, rb, s);
+          hit = i < rb && paged_read(P, rtable, i) == s;
+        } else {
+          const int i = lower_bound_dev(P.adj + b0, (int)len, s);
+          hit = i < len && __ldg(P.adj + b0 + i) == s;
+        }
+      }
+    }
+    const long long total = len - __popc(__ballot_sync(FULL, hit));
+    if (STATS && lane == d) c.lnodes += (unsigned long long)total;
+    return total;
+  }
+
+  // the streamed operand A: the reused list, else the shortest windowed adjacency list
+  int tA = -1;
+  long long bA, eA;
+  if (r >= 0) {
+    bA = ra;
+    eA = rb;
+  } else {
+    const long long len = (lane < nops) ? (oe - ob) : LLONG_MAX;
+    const unsigned minlen = __reduce_min_sync(FULL, (unsigned)min(len, (long long)UINT_MAX));
+    if (minlen == 0) return 0;
+    tA = __ffs(__ballot_sync(FULL, lane < nops && (unsigned)len == minlen)) - 1;
+    bA = __shfl_sync(FULL, ob, tA);
+    eA = __shfl_sync(FULL, oe, tA);
+  }
+  if (r >= 0 && nops > 0) {
+    const unsigned z = __ballot_sync(FULL, lane < nops && oe <= ob);
+    if (z) return 0;
+  }
+  const uint32_t others = __ballot_sync(FULL, lane < nops && lane != tA);
+  const int need_label = (r >= 0 && pl.label[r] == pl.label[d]) ? -1 : pl.label[d];
+  const int dmin = (r >= 0 && pl.deg_min[r] >= pl.deg_min[d]) ? 0 : pl.deg_min[d];
 
   PagedWriter w;
   w.table = c.tables + (size_t)(d - 2) * P.E;
@@ -128,22 +196,51 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d) {
   for (long long base = bA; base < eA; base += 32) {
     const long long i = base + lane;
     const bool inr = i < eA;
-    const int v = inr ? __ldg(P.adj + i) : INT_MAX;
+    int v = INT_MAX;
+    if (inr) v = (r >= 0) ? paged_read(P, rtable, i) : __ldg(P.adj + i);
     bool ok = inr;
     const int last_lane = (int)min(31ll, eA - 1 - base);
-    // probe the other operands (per-lane binary search, advancing lower bound)
+    // probe the other operands: merge (32-id register chunks, shuffle search) when the
+    // operand is at most kMergeRatio times longer than A, else per-lane binary search;
+    // either way the operand's lower bound advances batch by batch
     uint32_t om = others;
     while (om) {
       const int t = __ffs(om) - 1;
       om &= om - 1;
       const long long tb = __shfl_sync(FULL, ob, t);
       const long long te = __shfl_sync(FULL, oe, t);
-      int pos = (int)(te - tb);
-      const bool probe = inr && (ok || lane == last_lane);
-      if (probe) pos = lower_bound_dev(P.adj + tb, (int)(te - tb), v);
-      if (ok) ok = (pos < te - tb) && __ldg(P.adj + tb + pos) == v;
-      const int adv = __shfl_sync(FULL, pos, last_lane);
-      if (lane == t) ob = tb + adv;
+      const int th = __shfl_sync(FULL, hid, t);
+      if (th >= 0) {
+        // hub operand: one bitmap load per candidate (v is inside the window already)
+        if (ok) ok = (__ldg(P.hub_bits + (long long)th * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
+      } else if ((te - tb) <= (long long)P.merge_ratio * (eA - base)) {
+        // warp merge: walk B in coalesced 32-id chunks until a chunk reaches the batch max
+        const int amax = __shfl_sync(FULL, v, last_lane);
+        bool found = false;
+        long long ptr = tb;
+        while (ptr < te) {
+          const long long j = ptr + lane;
+          const int bv = (j < te) ? __ldg(P.adj + j) : INT_MAX;
+          int pos = 0;
+#pragma unroll
+          for (int s = 16; s > 0; s >>= 1)
+            if (__shfl_sync(FULL, bv, pos + s - 1) < v) pos += s;
+          found |= (__shfl_sync(FULL, bv, pos) == v);
+          const int bmax = __shfl_sync(FULL, bv, 31);
+          if (bmax >= amax) break;
+          ptr += 32;
+        }
+        ok = ok && found;
+        if (lane == t) ob = min(ptr, te);
+      } else {
+        int pos = (int)(te - tb);
+        const bool probe = inr && (ok || lane == last_lane);
+        if (probe) pos = P.bsearch_variant ? lower_bound_pow2(P.adj + tb, (int)(te - tb), v)
+                                           : lower_bound_dev(P.adj + tb, (int)(te - tb), v);
+        if (ok) ok = (pos < te - tb) && __ldg(P.adj + tb + pos) == v;
+        const int adv = __shfl_sync(FULL, pos, last_lane);
+        if (lane == t) ob = tb + adv;
+      }
       if (!__any_sync(FULL, ok)) break;
     }
     // fused filters: injectivity, label, degree
@@ -206,19 +303,20 @@ template <int MODE, bool STATS>
 __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) {
   const int k = P.plan.k;
   const int lane = c.lane;
+  const bool own2 = (start == 2);  // level 2 built by this warp (not a <v1,v2,v3> task)
   if (start == k - 1) {
-    long long n = (MODE == 1) ? extend<2, STATS>(P, c, start) : extend<1, STATS>(P, c, start);
+    long long n = (MODE == 1) ? extend<2, STATS>(P, c, start, own2) : extend<1, STATS>(P, c, start, own2);
     c.count += (unsigned long long)n;
     return true;
   }
   int d = start;
-  long long sz = extend<0, STATS>(P, c, d);
+  long long sz = extend<0, STATS>(P, c, d, own2);
   if (sz < 0) return false;
-  if (lane == d) { c.lsize = sz; c.liter = 0; }
+  if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
   bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
   for (;;) {
-    const long long it = __shfl_sync(FULL, c.liter, d);
-    const long long size = __shfl_sync(FULL, c.lsize, d);
+    const int it = __shfl_sync(FULL, c.liter, d);
+    const int size = __shfl_sync(FULL, c.lsize, d);
     if (it < size) {
       if (d == 2 && !grace && timed_out(P, c)) {
         // timeout: push the current and all remaining siblings, then backtrack
@@ -229,7 +327,7 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
           continue;
         }
         // queue full: the pushed prefix is gone, continue in place with t0 reset
-        if (lane == d) c.liter = upto;
+        if (lane == d) c.liter = (int)upto;
         if (lane == 0) c.t0 = globaltimer();
         grace = true;
         continue;
@@ -239,13 +337,13 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
       const int v = paged_read(P, table, it);
       if (lane == d) { c.sreg = v; c.liter = it + 1; }
       if (d + 1 == k - 1) {
-        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1) : extend<1, STATS>(P, c, d + 1);
+        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
         c.count += (unsigned long long)n;
       } else {
         d++;
-        sz = extend<0, STATS>(P, c, d);
+        sz = extend<0, STATS>(P, c, d, own2);
         if (sz < 0) return false;
-        if (lane == d) { c.lsize = sz; c.liter = 0; }
+        if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
       }
     } else {
       if (d == start) break;
@@ -329,7 +427,10 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
 
 // The persistent matching kernel.  MODE 0 = count, 1 = enumerate.
 template <int MODE, bool STATS>
-__global__ void __launch_bounds__(128, 8) tdfs_kernel(const KParams P) {
+#ifndef TDFS_MIN_BLOCKS
+#define TDFS_MIN_BLOCKS 16
+#endif
+__global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParams P) {
   const int lane = threadIdx.x & 31;
   const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   Ctx<STATS> c;
@@ -572,6 +673,12 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.label = g->d_label;
   P.n = g->n;
   P.plan = p->dev;
+  if (o->flags & TDFS_RUN_NO_REUSE) {
+    for (int i = 0; i < kMaxK; i++) { P.plan.reuse[i] = -1; P.plan.shortcut[i] &= 2; }
+    P.plan.reuse_enabled = 0;
+  }
+  if (o->flags & TDFS_RUN_NO_SHORTCUT)
+    for (int i = 0; i < kMaxK; i++) P.plan.shortcut[i] = 0;
   P.shard_rank = o->shard_rank;
   P.shard_world = o->shard_world;
   P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
@@ -587,6 +694,15 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.page_shift = L.page_shift;
   P.E = L.E;
   P.tau_ns = o->tau_ns;
+  P.merge_ratio = kMergeRatio;
+  if (const char* e = getenv("TDFS_MERGE_RATIO")) P.merge_ratio = atoi(e);  // tuning knob (experiments)
+  P.bsearch_variant = 0;
+  if (g->d_hub_bits && !(o->flags & TDFS_RUN_NO_HUB_BITMAP)) {
+    P.hub_id = g->d_hub_id;
+    P.hub_bits = g->d_hub_bits;
+    P.hub_words = g->hub_words;
+  }
+  if (const char* e = getenv("TDFS_BSEARCH")) P.bsearch_variant = atoi(e);
   P.out = d_out;
   P.cap = cap;
   int32_t* d_trace = nullptr;

@@ -129,6 +129,41 @@ void build_dev(const QueryAdj& q, Plan& P) {
     int nb = __builtin_popcount(d.bwd[p]);
     d.deg_min[p] = (p <= 1 || dq > nb) ? dq : 0;
   }
+  // Set-intersection result reuse: position p may start from the stored
+  // candidate list C(r) of an earlier position r when B(r) is a subset of B(p) -- and, because
+  // C(r) is already filtered, when every filter applied at r also holds for p's candidates:
+  // same (or no) label, r's degree threshold implied at p, r's constraint window implied at p.
+  // Largest B(r) wins (most operands saved), then the latest r.
+  for (int p = 0; p < kMaxK; p++) { d.reuse[p] = -1; d.shortcut[p] = 0; }
+  for (int p = 3; p < q.k; p++) {
+    int best = -1;
+    for (int r = 2; r < p && r <= q.k - 2; r++) {
+      if ((d.bwd[r] & d.bwd[p]) != d.bwd[r]) continue;
+      if (d.label[r] >= 0 && d.label[r] != d.label[p]) continue;
+      int nb = __builtin_popcount(d.bwd[p]);
+      if (d.deg_min[r] > std::max(d.deg_min[p], nb)) continue;
+      if ((d.lo_mask[r] & d.lo_mask[p]) != d.lo_mask[r]) continue;
+      if ((d.hi_mask[r] & d.hi_mask[p]) != d.hi_mask[r]) continue;
+      if (best < 0 || __builtin_popcount(d.bwd[r]) >= __builtin_popcount(d.bwd[best])) best = r;
+    }
+    d.reuse[p] = (int8_t)best;
+  }
+  // Count-only last position: when one list remains (one backward operand, or a reused C(r)
+  // with B(r) = B(p)) and no per-element label/degree test is needed, |C(p)| is the size of
+  // the constraint window minus the already-matched vertices inside it (no scan).
+  {
+    int p = q.k - 1;
+    if (p >= 2) {
+      int nb = __builtin_popcount(d.bwd[p]);
+      bool nolab = d.label[p] < 0, nodeg = d.deg_min[p] == 0;
+      if (nb == 1 && nolab && nodeg) d.shortcut[p] |= 2;
+      int r = d.reuse[p];
+      if (r >= 0 && d.bwd[r] == d.bwd[p] && (nolab || d.label[r] == d.label[p]) &&
+          (nodeg || d.deg_min[r] >= d.deg_min[p]))
+        d.shortcut[p] |= 1;
+    }
+  }
+  d.reuse_enabled = 1;
 }
 
 }  // namespace

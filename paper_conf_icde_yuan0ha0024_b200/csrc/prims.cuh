@@ -4,6 +4,7 @@
 #pragma once
 
 constexpr unsigned FULL = 0xffffffffu;
+constexpr long long kMergeRatio = 4;  // Eq. (1) probe: merge when |B| <= 4 |A remaining|, else binary search
 constexpr uint32_t NULL_PAGE = 0xffffffffu;
 constexpr int ERR_STACK = 1;
 
@@ -51,11 +52,11 @@ __device__ __forceinline__ void raise_error(const KParams& P, int code) {
   atomicCAS(reinterpret_cast<unsigned long long*>(ctr(P, C_ERROR)), 0ull, (unsigned long long)code);
 }
 
-// lower_bound of v in B[0, n) (sorted), n < 2^31
+// lower_bound of v in B[0, n) (sorted), n < 2^31 (halving search).
 __device__ __forceinline__ int lower_bound_dev(const int32_t* __restrict__ B, int n, int v) {
   int base = 0;
   while (n > 0) {
-    int half = n >> 1;
+    const int half = n >> 1;
     if (__ldg(B + base + half) < v) {
       base += half + 1;
       n -= half + 1;
@@ -64,6 +65,17 @@ __device__ __forceinline__ int lower_bound_dev(const int32_t* __restrict__ B, in
     }
   }
   return base;
+}
+
+// Same result with power-of-two steps (trip count depends only on n: no divergence).
+__device__ __forceinline__ int lower_bound_pow2(const int32_t* __restrict__ B, int n, int v) {
+  if (n <= 0) return 0;
+  int pos = 0;
+  for (int step = 1 << (31 - __clz(n)); step > 0; step >>= 1) {
+    const int q = pos + step;
+    if (q <= n && __ldg(B + q - 1) < v) pos = q;
+  }
+  return pos;
 }
 
 // ------------------------------------------------------------ Q_task (Alg. 3)

@@ -1,0 +1,16 @@
+#!/bin/bash
+# One GPU round-trip: full -m gpu suite, then a bench line (no cpu baseline).
+export PYTHONPATH=$PWD
+TAG=${1:-x}
+timeout 1500 python -m pytest tests -m gpu -q -x --timeout 400 --timeout-method=thread -p no:cacheprovider 2>&1 \
+  | grep -v "^  File\|^    " | tail -25 > gpurun_out/gputests_${TAG}.log
+cat gpurun_out/gputests_${TAG}.log
+timeout 900 python bench.py --steps 3 --warmup 3 --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
+tail -2 gpurun_out/bench_${TAG}.err
+python - <<PY
+import json
+d = json.load(open("gpurun_out/bench_${TAG}.json"))
+print("value %.4g  ms/step %.1f  frac %.3f  e2e %.4g" % (d["value"], d["ms_per_step"], d["roofline"]["frac"], (d["e2e"] or {}).get("value", 0)))
+for k, v in d["config"]["per_query"].items():
+    print("  %-16s %10.2f ms  %d" % (k, v["time_to_count_ms"], v["count"]))
+PY

@@ -141,6 +141,40 @@ def test_tau_and_page_invariance(tau_ms, page_bytes):
         assert got == ref, (name, tau_ms, page_bytes)
 
 
+@pytest.mark.parametrize("flags", [0, 4, 8, 12])
+def test_reuse_and_shortcut_invariance(flags):
+    """Set-intersection result reuse and the count-only last level never
+    change results: counts and per-level node counts equal the oracle with every flag combination."""
+    g = graph("r10")
+    for name in ["k4", "diamond", "tailed_triangle", "house", "k5", "prism", "w5", "fig1_q", "wedge", "star3"]:
+        q = T.query(name)
+        order = O.oracle_order(q)
+        cnt, st = U.count(g, q, "auto", order=order, stats=True, flags=flags)
+        r = O.match(g, q, "auto", order=order, deg_filter=True, threads=THREADS)
+        assert cnt == r["count"], (name, flags)
+        assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k], (name, flags)
+        assert U.count(g, q, "auto", flags=flags) == r["count"], (name, flags)
+    for name in ["k4", "diamond", "two_k4"]:
+        q = T.labeled_query(name, 2)
+        gl = graph("r10").with_labels(2, 5)
+        assert U.count(gl, q, "auto", flags=flags) == O.count(gl, q, "auto", threads=THREADS), (name, flags)
+
+
+def test_hub_bitmaps_do_not_change_results():
+    """Hub adjacency bitmaps (degree >= 256) replace binary searches; results are identical."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    g = T.rmat(12, 24, 5)
+    assert int(np.bincount(g.edges.reshape(-1)).max()) >= 256
+    for name in ["triangle", "k4"]:
+        q = T.query(name)
+        ref = O.count(g, q, "auto", threads=THREADS)
+        assert U.count(g, q, "auto") == ref
+        assert U.count(g, q, "auto", flags=M.TDFS_RUN_NO_HUB_BITMAP) == ref
+    for name in ["c4", "diamond", "tailed_triangle", "house"]:
+        q = T.query(name)
+        assert U.count(g, q, "auto") == U.count(g, q, "auto", flags=M.TDFS_RUN_NO_HUB_BITMAP | 4 | 8), name
+
+
 def test_chunk_queue_grid_invariance():
     rmat12 = graph("r10")
     q = T.query("house")
