@@ -221,10 +221,11 @@ def run_ours(a):
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{dev}")
 
     # W (algorithmic adjacency bytes) per query from one instrumented run (untimed)
-    W, stats_runs = [], []
+    W, Wfull, stats_runs = [], [], []
     for p in plans:
         c, st = M.tdfs_count(h, p, opts, workspace=ws, stats=True)
-        W.append(st["adj_bytes"])
+        W.append(st["stream_bytes"])   # roofline bytes, R29b
+        Wfull.append(st["adj_bytes"])  # SURVEY 8(d) full-operand W, for reference
         stats_runs.append(st)
 
     def step(ev_q=None):
@@ -338,7 +339,8 @@ def run_ours(a):
         for i, q in enumerate(qs):
             per_query[q.name] = {"count": int(counts[i]), "time_to_count_ms": q_tot[i] / a.steps,
                                  "matches_per_s": counts[i] / (q_tot[i] / a.steps / 1000.0),
-                                 "W_bytes": int(W[i]), "eff_GBps": W[i] / (q_tot[i] / a.steps / 1000.0) / 1e9,
+                                 "W_bytes": int(W[i]), "W_full_bytes": int(Wfull[i]),
+                                 "eff_GBps": W[i] / (q_tot[i] / a.steps / 1000.0) / 1e9,
                                  "timeouts": int(stats_runs[i]["timeouts"]),
                                  "tasks_enqueued": int(stats_runs[i]["tasks_enqueued"]),
                                  "pages_used": int(stats_runs[i]["pages_used"])}
@@ -354,8 +356,10 @@ def run_ours(a):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_kind": peak_kind,
-                         "note": "achieved = algorithmic adjacency bytes W (SURVEY 8(d)) per matching-kernel launch "
-                                 "/ average tdfs_count duration (CUDA events on the launch stream)"},
+                         "note": "achieved = algorithmic bytes per matching-kernel launch (DESIGN.md R29b: 16 B per "
+                                 "Eq.(1) operand + 4 B x smallest constraint-windowed operand, per extension; from one "
+                                 "STATS run) / mean tdfs_count duration (CUDA events on the launch stream); traffic = "
+                                 "ncu dram bytes per launch (profiles/ncu_full_summary.json)"},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": 4 * len(qs) * a.steps,

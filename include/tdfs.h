@@ -174,6 +174,9 @@ typedef struct {
   float kernel_ms;            /* CUDA-event time of the matching kernel */
   int32_t grid_blocks, warps_per_block, page_table_entries, pad_;
   uint64_t pool_pages;
+  uint64_t stream_bytes;      /* roofline bytes (R29b): sum over extensions of 16 B per Eq. (1)
+                                 operand + 4 B x |smallest constraint-windowed operand| (0 for a count-only
+                                 last position with one operand and no label test) */
 } tdfs_stats;
 
 /* Bytes of caller-owned device workspace needed for one job (256-byte aligned). */

@@ -56,7 +56,7 @@ def _o():
                                      ctypes.c_int, I32P, I32P, ctypes.c_int,
                                      ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_int64,
                                      ctypes.c_int, ctypes.c_int64, I32P,
-                                     U64P, U64P, U64P]
+                                     U64P, U64P, U64P, U64P]
         lib.oracle_order.restype = ctypes.c_int
         lib.oracle_order.argtypes = [ctypes.c_int, ctypes.c_int, I32P, I32P]
         lib.oracle_automorphisms.restype = ctypes.c_int
@@ -120,6 +120,7 @@ def match(graph, query, constraints="auto", order: Optional[Sequence[int]] = Non
     cnt = ctypes.c_uint64(0)
     nodes = np.zeros(9, dtype=np.uint64)
     w = ctypes.c_uint64(0)
+    sb = ctypes.c_uint64(0)
     out = np.zeros(max(1, enumerate_cap) * q.k, dtype=np.int32) if enumerate_cap > 0 else None
     rlo, rhi = (0, -1) if roots is None else roots
     rc = _o().oracle_match(g.n, g.m, _p(eu, I32P), _p(ev, I32P), _p(lab, U8P),
@@ -127,10 +128,11 @@ def match(graph, query, constraints="auto", order: Optional[Sequence[int]] = Non
                            len(cons), _p(ca, I32P), _p(oa, I32P), int(bool(deg_filter)),
                            int(shard[0]), int(shard[1]), int(rlo), int(rhi),
                            int(threads), int(enumerate_cap), _p(out, I32P),
-                           ctypes.byref(cnt), nodes.ctypes.data_as(U64P), ctypes.byref(w))
+                           ctypes.byref(cnt), nodes.ctypes.data_as(U64P), ctypes.byref(w), ctypes.byref(sb))
     if rc < 0:
         raise ValueError("oracle_match: bad arguments")
     res = {"count": int(cnt.value), "nodes": [int(x) for x in nodes[: q.k]], "W": int(w.value),
+           "W_stream": int(sb.value),
            "tuples": None, "overflow": rc == 1}
     if enumerate_cap > 0:
         n = min(res["count"], enumerate_cap)

@@ -40,6 +40,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstdint>
+#include <climits>
 #include <cstring>
 #include <mutex>
 #include <thread>
@@ -78,6 +79,7 @@ struct Acc {
   uint64_t count = 0;
   uint64_t nodes[9] = {0};
   uint64_t wbytes = 0;
+  uint64_t sbytes = 0;   /* R29b */
   std::vector<int32_t> tuples;  // local tuples (enumerate)
 };
 
@@ -148,6 +150,23 @@ void enumerate(const Job& J, std::vector<int32_t>& S, int i, Acc& acc,
   const std::vector<int32_t>& C = *candidates(J, S, i, cbuf[i]);  /* line 3 */
   if (i >= 2) {                                        /* W of SURVEY 8(d) */
     for (int pj : J.bwd[i]) acc.wbytes += 4ull * (uint64_t)degree(*J.g, S[pj]) + 16ull;
+    /* R29b: 16 B per operand + 4 B x the smallest operand restricted to the ids the
+     * constraints already allow (lo <= w < hi); nothing for a count-only last position
+     * with a single operand and no label test */
+    int64_t lo = 0, hi = (int64_t)INT32_MAX + 1;
+    for (auto& c : J.cons_at[i]) {
+      if (c.second > 0) lo = std::max<int64_t>(lo, (int64_t)S[c.first] + 1);
+      else hi = std::min<int64_t>(hi, (int64_t)S[c.first]);
+    }
+    uint64_t mn = UINT64_MAX;
+    for (int pj : J.bwd[i]) {
+      const auto& L = J.g->adj[S[pj]];
+      uint64_t len = 0;
+      if (lo < hi) len = (uint64_t)(std::lower_bound(L.begin(), L.end(), hi) - std::lower_bound(L.begin(), L.end(), lo));
+      mn = std::min(mn, len);
+    }
+    bool count_only = (i + 1 == J.q->k) && J.bwd[i].size() == 1 && J.q->label[J.order[i]] < 0;
+    acc.sbytes += 16ull * J.bwd[i].size() + ((count_only || lo >= hi || mn == UINT64_MAX) ? 0ull : 4ull * mn);
   }
   for (size_t t = 0; t < C.size(); t++) {              /* line 4 */
     int32_t v = C[t];
@@ -255,7 +274,7 @@ int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, con
                  int nc, const int32_t* cons, const int32_t* order, int deg_filter,
                  int shard_rank, int shard_world, int64_t root_lo, int64_t root_hi,
                  int nthreads, int64_t max_out, int32_t* out_tuples,
-                 uint64_t* out_count, uint64_t* out_nodes, uint64_t* out_w) {
+                 uint64_t* out_count, uint64_t* out_nodes, uint64_t* out_w, uint64_t* out_stream) {
   QueryGraph q;
   if (!build_query(k, nqe, qedges, qlabels, nc, cons, q)) return -1;
   if (shard_world < 1 || shard_rank < 0 || shard_rank >= shard_world) return -1;
@@ -330,14 +349,16 @@ int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, con
     for (int t = 0; t < nthreads; t++) th.emplace_back(worker, t);
     for (auto& x : th) x.join();
   }
-  uint64_t count = 0, w = 0, nodes[9] = {0};
+  uint64_t count = 0, w = 0, sb = 0, nodes[9] = {0};
   for (auto& a : accs) {
     count += a.count;
     w += a.wbytes;
+    sb += a.sbytes;
     for (int i = 0; i < 9; i++) nodes[i] += a.nodes[i];
   }
   if (out_count) *out_count = count;
   if (out_w) *out_w = w;
+  if (out_stream) *out_stream = sb;
   if (out_nodes)
     for (int i = 0; i < k; i++) out_nodes[i] = nodes[i];
   int rc = 0;

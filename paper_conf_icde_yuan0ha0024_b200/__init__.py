@@ -79,7 +79,7 @@ class tdfs_stats(ctypes.Structure):
                 ("edges_scanned", ctypes.c_uint64), ("edges_filtered_in", ctypes.c_uint64),
                 ("chunks_fetched", ctypes.c_uint64), ("kernel_ms", ctypes.c_float), ("grid_blocks", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("page_table_entries", ctypes.c_int32), ("pad_", ctypes.c_int32),
-                ("pool_pages", ctypes.c_uint64)]
+                ("pool_pages", ctypes.c_uint64), ("stream_bytes", ctypes.c_uint64)]
 
     def as_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f not in ("nodes_per_level", "pad_")}

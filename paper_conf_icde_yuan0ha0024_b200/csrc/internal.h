@@ -75,7 +75,7 @@ constexpr int kCounterStride = 16;  // u64 words per counter (128 B)
 
 enum StatIdx {
   S_NODES = 0,                 // 9 entries
-  S_ADJ_BYTES = 9, S_ENQ, S_DEQ, S_TIMEOUTS, S_QFULL, S_EDGES_SCANNED, S_EDGES_IN, S_CHUNKS,
+  S_ADJ_BYTES = 9, S_ENQ, S_DEQ, S_TIMEOUTS, S_QFULL, S_EDGES_SCANNED, S_EDGES_IN, S_CHUNKS, S_STREAM,
   S_NUM
 };
 

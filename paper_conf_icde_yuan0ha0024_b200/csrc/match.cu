@@ -52,7 +52,7 @@ struct Ctx {
   unsigned long long count;  // warp-uniform
   unsigned long long t0;     // lane 0: task start time
   unsigned long long lnodes; // lane p: nodes[p]   (STATS)
-  unsigned long long wbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
+  unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
 };
 
@@ -120,6 +120,21 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
   const int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
   const int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
+  if (STATS) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
+    const bool mine = (bm_all >> lane) & 1u;
+    unsigned wlen = UINT_MAX;
+    if (mine && lo < hi) {
+      const long long b = __ldg(P.offs + c.sreg), e = __ldg(P.offs + c.sreg + 1);
+      const int n = (int)(e - b);
+      const int a = lo > 0 ? lower_bound_dev(P.adj + b, n, lo) : 0;
+      const int z = hi < INT_MAX ? a + lower_bound_dev(P.adj + b + a, n - a, hi) : n;
+      wlen = (unsigned)(z - a);
+    }
+    const unsigned mn = __reduce_min_sync(FULL, wlen);
+    const int nall = __popc(bm_all);
+    const bool count_only = (d == pl.k - 1) && nall == 1 && pl.label[d] < 0 && pl.deg_min[d] == 0;
+    if (lane == 0) c.sbytes += 16ull * nall + ((lo >= hi || count_only || mn == UINT_MAX) ? 0ull : 4ull * mn);
+  }
   if (lo >= hi) return 0;
   const bool windowed = (lo > 0 || hi < INT_MAX);
   if (lane < nops && windowed) {
@@ -441,7 +456,7 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.count = 0;
   c.t0 = 0;
   c.lnodes = 0;
-  c.wbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
+  c.wbytes = c.sbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
   const Queue q = make_queue(P);
   int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
@@ -524,6 +539,7 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
     if (lane < kMaxK + 1 && c.lnodes) atomicAdd(P.stats + S_NODES + lane, c.lnodes);
     if (lane == 0) {
       atomicAdd(P.stats + S_ADJ_BYTES, c.wbytes);
+      atomicAdd(P.stats + S_STREAM, c.sbytes);
       atomicAdd(P.stats + S_ENQ, c.enq);
       atomicAdd(P.stats + S_DEQ, c.deq);
       atomicAdd(P.stats + S_TIMEOUTS, c.touts);
@@ -768,6 +784,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     stats->chunks_fetched = hs[S_CHUNKS];
     stats->pages_used = std::min<unsigned long long>(hc[C_POOL * kCounterStride], L.n_pages);
     stats->pool_pages = L.n_pages;
+    stats->stream_bytes = hs[S_STREAM];
     stats->grid_blocks = L.blocks;
     stats->warps_per_block = L.wpb;
     stats->page_table_entries = L.E;

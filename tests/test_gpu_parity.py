@@ -235,6 +235,7 @@ def test_nodes_per_level_and_W_match_oracle(name):
         assert cnt == r["count"]
         assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k]
         assert st["adj_bytes"] == r["W"]
+        assert st["stream_bytes"] == r["W_stream"]
 
 
 def test_stack_exhaustion_is_an_error_never_a_count():

@@ -268,6 +268,25 @@ def test_nodes_and_W_triangle_closed_form():
     assert r["nodes"][2] == r["count"]
 
 
+def test_W_stream_triangle_closed_form():
+    """R29b roofline bytes for the triangle, order [0,1,2], constraints 0<1<2: each internal
+    prefix (edge u<v, both degrees >= 2) adds 2 x 16 B + 4 B x min(|N(u) > v|, |N(v) > v|)."""
+    g = T.rmat(10, 8, 13)
+    d = _degrees(g)
+    nbrs = [[] for _ in range(g.n)]
+    for a, b in g.edges.tolist():
+        nbrs[a].append(b)
+        nbrs[b].append(a)
+    tot = 0
+    for u, v in g.edges.tolist():
+        if d[u] >= 2 and d[v] >= 2:
+            tot += 32 + 4 * min(sum(1 for w in nbrs[u] if w > v), sum(1 for w in nbrs[v] if w > v))
+    assert O.match(g, T.query("triangle"), "auto", order=[0, 1, 2])["W_stream"] == tot
+    # a count-only single-operand last position streams nothing: wedge = 16 B per prefix
+    r = O.match(g, T.query("wedge"), "auto", order=[0, 1, 2])
+    assert r["W_stream"] == 16 * r["nodes"][1]
+
+
 def test_enumerate_tuples_satisfy_definition():
     g = T.rmat(8, 6, 21)
     q = T.query("house")
