@@ -57,6 +57,16 @@ def _o():
                                      ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_int64,
                                      ctypes.c_int, ctypes.c_int64, I32P,
                                      U64P, U64P, U64P, U64P]
+        lib.oracle_graph_new.restype = ctypes.c_void_p
+        lib.oracle_graph_new.argtypes = [ctypes.c_int64, ctypes.c_int64, I32P, I32P, U8P]
+        lib.oracle_graph_free.restype = None
+        lib.oracle_graph_free.argtypes = [ctypes.c_void_p]
+        lib.oracle_match_g.restype = ctypes.c_int
+        lib.oracle_match_g.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, I32P, I32P,
+                                       ctypes.c_int, I32P, I32P, ctypes.c_int,
+                                       ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_int64,
+                                       ctypes.c_int, ctypes.c_int64, I32P,
+                                       U64P, U64P, U64P, U64P]
         lib.oracle_order.restype = ctypes.c_int
         lib.oracle_order.argtypes = [ctypes.c_int, ctypes.c_int, I32P, I32P]
         lib.oracle_automorphisms.restype = ctypes.c_int
@@ -103,14 +113,31 @@ def _constraints(query, constraints) -> List[Tuple[int, int]]:
     return [(int(a), int(b)) for a, b in constraints]
 
 
+class OracleGraph:
+    """The oracle's adjacency built once for many queries (large configs)."""
+
+    def __init__(self, graph):
+        self.graph = graph
+        g = graph
+        eu = _i32(g.edges[:, 0]) if g.m else np.zeros(1, np.int32)
+        ev = _i32(g.edges[:, 1]) if g.m else np.zeros(1, np.int32)
+        self._lab = None if g.labels is None else np.ascontiguousarray(g.labels, dtype=np.uint8)
+        self.ptr = _o().oracle_graph_new(g.n, g.m, _p(eu, I32P), _p(ev, I32P), _p(self._lab, U8P))
+
+    def __del__(self):
+        try:
+            if self.ptr:
+                _o().oracle_graph_free(self.ptr)
+                self.ptr = None
+        except Exception:
+            pass
+
+
 def match(graph, query, constraints="auto", order: Optional[Sequence[int]] = None, deg_filter: bool = True,
           shard: Tuple[int, int] = (0, 1), roots: Optional[Tuple[int, int]] = None, threads: int = 1,
           enumerate_cap: int = 0):
-    """Run O2.  Returns dict(count, nodes (list, k), W, tuples (ndarray or None), overflow)."""
-    g = graph
-    eu = _i32(g.edges[:, 0]) if g.m else np.zeros(1, np.int32)
-    ev = _i32(g.edges[:, 1]) if g.m else np.zeros(1, np.int32)
-    lab = None if g.labels is None else np.ascontiguousarray(g.labels, dtype=np.uint8)
+    """Run O2 on a tdfs_inputs.Graph or an OracleGraph.
+    Returns dict(count, nodes (list, k), W, W_stream, tuples (ndarray or None), overflow)."""
     q = query
     qe = _i32(q.edges).reshape(-1)
     ql = None if q.labels is None else _i32(q.labels)
@@ -123,17 +150,23 @@ def match(graph, query, constraints="auto", order: Optional[Sequence[int]] = Non
     sb = ctypes.c_uint64(0)
     out = np.zeros(max(1, enumerate_cap) * q.k, dtype=np.int32) if enumerate_cap > 0 else None
     rlo, rhi = (0, -1) if roots is None else roots
-    rc = _o().oracle_match(g.n, g.m, _p(eu, I32P), _p(ev, I32P), _p(lab, U8P),
-                           q.k, len(q.edges), _p(qe, I32P), _p(ql, I32P),
-                           len(cons), _p(ca, I32P), _p(oa, I32P), int(bool(deg_filter)),
-                           int(shard[0]), int(shard[1]), int(rlo), int(rhi),
-                           int(threads), int(enumerate_cap), _p(out, I32P),
-                           ctypes.byref(cnt), nodes.ctypes.data_as(U64P), ctypes.byref(w), ctypes.byref(sb))
+    tail = (len(cons), _p(ca, I32P), _p(oa, I32P), int(bool(deg_filter)),
+            int(shard[0]), int(shard[1]), int(rlo), int(rhi),
+            int(threads), int(enumerate_cap), _p(out, I32P),
+            ctypes.byref(cnt), nodes.ctypes.data_as(U64P), ctypes.byref(w), ctypes.byref(sb))
+    if isinstance(graph, OracleGraph):
+        rc = _o().oracle_match_g(graph.ptr, q.k, len(q.edges), _p(qe, I32P), _p(ql, I32P), *tail)
+    else:
+        g = graph
+        eu = _i32(g.edges[:, 0]) if g.m else np.zeros(1, np.int32)
+        ev = _i32(g.edges[:, 1]) if g.m else np.zeros(1, np.int32)
+        lab = None if g.labels is None else np.ascontiguousarray(g.labels, dtype=np.uint8)
+        rc = _o().oracle_match(g.n, g.m, _p(eu, I32P), _p(ev, I32P), _p(lab, U8P),
+                               q.k, len(q.edges), _p(qe, I32P), _p(ql, I32P), *tail)
     if rc < 0:
         raise ValueError("oracle_match: bad arguments")
     res = {"count": int(cnt.value), "nodes": [int(x) for x in nodes[: q.k]], "W": int(w.value),
-           "W_stream": int(sb.value),
-           "tuples": None, "overflow": rc == 1}
+           "W_stream": int(sb.value), "tuples": None, "overflow": rc == 1}
     if enumerate_cap > 0:
         n = min(res["count"], enumerate_cap)
         res["tuples"] = out[: n * q.k].reshape(n, q.k).copy()

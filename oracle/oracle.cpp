@@ -269,7 +269,7 @@ extern "C" {
  * Returns 0 on success, -1 on bad arguments, 1 if more than max_out tuples
  * exist (count still exact; first max_out tuples in DFS order written).
  */
-int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, const uint8_t* label,
+static int match_on(const DataGraph& g,
                  int k, int nqe, const int32_t* qedges, const int32_t* qlabels,
                  int nc, const int32_t* cons, const int32_t* order, int deg_filter,
                  int shard_rank, int shard_world, int64_t root_lo, int64_t root_hi,
@@ -278,9 +278,7 @@ int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, con
   QueryGraph q;
   if (!build_query(k, nqe, qedges, qlabels, nc, cons, q)) return -1;
   if (shard_world < 1 || shard_rank < 0 || shard_rank >= shard_world) return -1;
-  DataGraph g;
-  build_data(n, m, eu, ev, label, g);
-
+  const int64_t n = g.n;
   Job J;
   J.g = &g;
   J.q = &q;
@@ -370,6 +368,36 @@ int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, con
     if (have > max_out) rc = 1;
   }
   return rc;
+}
+
+int oracle_match(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, const uint8_t* label,
+                 int k, int nqe, const int32_t* qedges, const int32_t* qlabels,
+                 int nc, const int32_t* cons, const int32_t* order, int deg_filter,
+                 int shard_rank, int shard_world, int64_t root_lo, int64_t root_hi,
+                 int nthreads, int64_t max_out, int32_t* out_tuples,
+                 uint64_t* out_count, uint64_t* out_nodes, uint64_t* out_w, uint64_t* out_stream) {
+  DataGraph g;
+  build_data(n, m, eu, ev, label, g);
+  return match_on(g, k, nqe, qedges, qlabels, nc, cons, order, deg_filter, shard_rank, shard_world, root_lo, root_hi,
+                  nthreads, max_out, out_tuples, out_count, out_nodes, out_w, out_stream);
+}
+
+/* Build the oracle's adjacency once and run many queries on it (same semantics). */
+void* oracle_graph_new(int64_t n, int64_t m, const int32_t* eu, const int32_t* ev, const uint8_t* label) {
+  DataGraph* g = new DataGraph;
+  build_data(n, m, eu, ev, label, *g);
+  return g;
+}
+
+void oracle_graph_free(void* g) { delete (DataGraph*)g; }
+
+int oracle_match_g(const void* g, int k, int nqe, const int32_t* qedges, const int32_t* qlabels,
+                   int nc, const int32_t* cons, const int32_t* order, int deg_filter,
+                   int shard_rank, int shard_world, int64_t root_lo, int64_t root_hi,
+                   int nthreads, int64_t max_out, int32_t* out_tuples,
+                   uint64_t* out_count, uint64_t* out_nodes, uint64_t* out_w, uint64_t* out_stream) {
+  return match_on(*(const DataGraph*)g, k, nqe, qedges, qlabels, nc, cons, order, deg_filter, shard_rank, shard_world,
+                  root_lo, root_hi, nthreads, max_out, out_tuples, out_count, out_nodes, out_w, out_stream);
 }
 
 /* The oracle's own matching order (for reporting). */
