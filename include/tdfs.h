@@ -144,6 +144,7 @@ void tdfs_free_plan(tdfs_plan* p);
 #define TDFS_RUN_NO_REUSE 4u        /* ablation: disable set-intersection result reuse */
 #define TDFS_RUN_NO_SHORTCUT 8u     /* ablation: always scan the last level (no count-only window shortcut) */
 #define TDFS_RUN_NO_HUB_BITMAP 16u  /* ablation: probe hub adjacency lists by search, not by bitmap */
+#define TDFS_RUN_NO_LEAF_STAGE 32u  /* ablation: no shared-memory staging of the last position's fixed part */
 
 typedef struct {
   int64_t tau_ns;              /* timeout tau; default 10 ms;

@@ -20,19 +20,33 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // Per matching-order position p (pi_p = order[p]) everything the kernel needs,
 // precomputed on the host (PAPER.md:77 backward neighbours, :29 constraints,
 // :400 degree/label filters).  Bit j of a mask refers to position j < p.
+// Index kVF of the per-position arrays is a VIRTUAL position: the part of the last
+// position's Eq. (1) that does not depend on S[k-2] -- the "fixed" operands
+// B(u_{k-1}) restricted to positions <= k-3, the constraint windows and injectivity
+// tests against those positions, and the label/degree filters.  Its result F is
+// the same for every sibling at level k-2, so it is computed once per level-(k-2)
+// list and staged in shared memory; each leaf is then
+// |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
+constexpr int kVF = kMaxK;
+constexpr int kLeafStage = 512;  // default shared-memory ids per warp for the leaf set F
 struct DevPlan {
   int32_t k;
-  int32_t order[kMaxK];      // query vertex at position p (enumerate output mapping)
-  uint32_t bwd[kMaxK];       // B^pi(pi_p) as a position mask
-  uint32_t lo_mask[kMaxK];   // j with constraint f(pi_j) < f(pi_p): v > S[j]
-  uint32_t hi_mask[kMaxK];   // j with constraint f(pi_p) < f(pi_j): v < S[j]
-  uint32_t inj_mask[kMaxK];  // j whose v != S[j] is not implied by adjacency or a constraint
-  int32_t label[kMaxK];      // required label, -1 = any
-  int32_t deg_min[kMaxK];    // degree filter threshold (0 = off), R8
-  int32_t edge_cons;         // constraint between positions 0 and 1: +1 S0<S1, -1 S1<S0, 0 none
-  int32_t reuse_enabled;     // set-intersection result reuse on
-  int8_t reuse[kMaxK];       // stored position r whose candidate list C(r) is a superset start for p, -1 none
-  uint8_t shortcut[kMaxK];   // last position: count without scanning; bit0 valid with reuse, bit1 without
+  int32_t order[kMaxK];          // query vertex at position p (enumerate output mapping)
+  uint32_t bwd[kMaxK + 1];       // B^pi(pi_p) as a position mask
+  uint32_t lo_mask[kMaxK + 1];   // j with constraint f(pi_j) < f(pi_p): v > S[j]
+  uint32_t hi_mask[kMaxK + 1];   // j with constraint f(pi_p) < f(pi_j): v < S[j]
+  uint32_t inj_mask[kMaxK + 1];  // j whose v != S[j] is not implied by adjacency or a constraint
+  int32_t label[kMaxK + 1];      // required label, -1 = any
+  int32_t deg_min[kMaxK + 1];    // degree filter threshold (0 = off), R8
+  int32_t edge_cons;             // constraint between positions 0 and 1: +1 S0<S1, -1 S1<S0, 0 none
+  int32_t reuse_enabled;         // set-intersection result reuse on
+  int8_t reuse[kMaxK + 1];       // stored position r whose candidate list C(r) is a superset start for p, -1 none
+  uint8_t shortcut[kMaxK + 1];   // last position: count without scanning; bit0 valid with reuse, bit1 without
+  // leaf staging (position k-1 split into the virtual position kVF and the S[k-2] part)
+  int8_t lf_on;                  // k >= 4 and B(u_{k-1}) has an operand at a position <= k-3
+  int8_t lf_var;                 // N(S[k-2]) is an operand of position k-1
+  int8_t lf_lo_var, lf_hi_var;   // window bound v > S[k-2] / v < S[k-2]
+  int8_t lf_inj_var;             // v != S[k-2] must be tested (not implied)
 };
 
 struct Plan {
@@ -107,6 +121,9 @@ struct KParams {
   int32_t E;                   // page-table entries per level
   int64_t tau_ns;              // < 0: infinity
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
+  int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
+  int32_t lf_cost_g;           // leaf staging cost model: one dependent global load in shared-memory steps
+  int32_t coop_window;         // constraint windows by warp-cooperative 32-ary search (else per-lane binary)
   int32_t bsearch_variant;     // 0 halving, 1 power-of-two (experiments)
   // hub bitmaps (nullptr when off)
   const int32_t* hub_id;
@@ -124,7 +141,7 @@ struct KParams {
 struct WsLayout {
   size_t ctr = 0, stats = 0, slots = 0, tables = 0, pool = 0, total = 0;
   uint64_t qcap = 0, n_pages = 0;
-  int32_t E = 0, page_shift = 0, n_levels = 0, blocks = 0, wpb = 0;
+  int32_t E = 0, page_shift = 0, n_levels = 0, blocks = 0, wpb = 0, fcap = 0;
 };
 
 int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayout* L);
@@ -132,7 +149,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
                int mode /*0 count, 1 enumerate*/, int32_t* d_out, uint64_t cap, uint64_t* d_count,
                bool sync, uint64_t* h_count, tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap,
                int64_t* n_trace);
-int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int* out);
+int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int* out);
 const Graph* graph_of(const tdfs_graph* g);
 const Plan* plan_of(const tdfs_plan* p);
 

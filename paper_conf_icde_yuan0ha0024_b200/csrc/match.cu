@@ -54,6 +54,7 @@ struct Ctx {
   unsigned long long lnodes; // lane p: nodes[p]   (STATS)
   unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
+  int* sF;                  // this warp's shared-memory stage for the leaf set F (P.fcap ints)
 };
 
 __device__ __forceinline__ int getS(int sreg, int p) { return __shfl_sync(FULL, sreg, p); }
@@ -78,9 +79,55 @@ __device__ __forceinline__ long long paged_lower_bound(const KParams& P, const u
   return lo;
 }
 
+// lower_bound of v in the shared-memory list F[lo, hi) (all lanes, same v: broadcast reads)
+__device__ __forceinline__ int smem_lower_bound(const int* F, int lo, int hi, int v) {
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (F[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// Warp-cooperative lower_bound of v in the sorted global list L[0, n): each round the 32
+// lanes sample the remaining range at 32 evenly spaced points (one load per lane) and keep
+// one stride, so a list of n ids takes ceil(log32 n) dependent loads instead of log2 n.
+__device__ __forceinline__ long long warp_lower_bound(const int32_t* __restrict__ L, long long n, int v, int lane) {
+  long long lo = 0;
+  while (n > 32) {
+    const long long step = (n + 31) >> 5;
+    const long long i = lo + (long long)(lane + 1) * step - 1;  // last id of stride `lane`
+    const bool less = i < lo + n && __ldg(L + i) < v;
+    const int c = __popc(__ballot_sync(FULL, less));             // strides entirely below v
+    lo += (long long)c * step;
+    n = min(step, n - (long long)c * step);
+  }
+  const bool less = lane < n && __ldg(L + lo + lane) < v;
+  return lo + __popc(__ballot_sync(FULL, less));
+}
+
+// Warp-cooperative lower_bound of v in the paged list [lo, hi) of a stored level (same
+// scheme as warp_lower_bound; each sample is a page-table load and a page load).
+__device__ __forceinline__ long long warp_paged_lower_bound(const KParams& P, const uint32_t* table, long long lo,
+                                                            long long hi, int v, int lane) {
+  long long n = hi - lo;
+  while (n > 32) {
+    const long long step = (n + 31) >> 5;
+    const long long i = lo + (long long)(lane + 1) * step - 1;
+    const bool less = i < lo + n && paged_read(P, table, i) < v;
+    const int c = __popc(__ballot_sync(FULL, less));
+    lo += (long long)c * step;
+    n = min(step, n - (long long)c * step);
+  }
+  const bool less = lane < n && paged_read(P, table, lo + lane) < v;
+  return lo + __popc(__ballot_sync(FULL, less));
+}
+
 // Candidate generation for position d (Eq. 1 + fused filters).
 // MODE_OUT: 0 = store into the paged level of d; 1 = count only (last position);
-//           2 = enumerate (last position).
+//           2 = enumerate (last position); 3 = stage into shared memory (d = kVF, the
+//           S[k-2]-independent part of the last position), or return -2 without
+//           writing when the streamed operand exceeds the stage (P.fcap ids).
 // allow_reuse2: the stored list of position 2 belongs to this prefix (false for tasks
 // <v1,v2,v3> taken from Q_task, whose level 2 was built by another warp).
 // Returns the number of candidates, or -1 on stack exhaustion.
@@ -109,7 +156,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     oe = __ldg(P.offs + sj + 1);
     if (P.hub_id) hid = __ldg(P.hub_id + sj);
   }
-  if (STATS) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
+  if (STATS && MODE_OUT != 3) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
     const bool mine = (bm_all >> lane) & 1u;
     unsigned long long wb = 0;
     if (mine) wb = (unsigned long long)(4 * (__ldg(P.offs + c.sreg + 1) - __ldg(P.offs + c.sreg)) + 16);
@@ -120,7 +167,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
   const int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
   const int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
-  if (STATS) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
+  if (STATS && MODE_OUT != 3) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
     const bool mine = (bm_all >> lane) & 1u;
     unsigned wlen = UINT_MAX;
     if (mine && lo < hi) {
@@ -137,7 +184,15 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   }
   if (lo >= hi) return 0;
   const bool windowed = (lo > 0 || hi < INT_MAX);
-  if (lane < nops && windowed) {
+  if (windowed && P.coop_window) {
+    // warp-cooperative window search, one operand at a time (ceil(log32 n) dependent loads)
+    for (int t = 0; t < nops; t++) {
+      const long long tb = __shfl_sync(FULL, ob, t), te = __shfl_sync(FULL, oe, t);
+      const long long a = lo > 0 ? warp_lower_bound(P.adj + tb, te - tb, lo, lane) : 0;
+      const long long b = hi < INT_MAX ? a + warp_lower_bound(P.adj + tb + a, te - tb - a, hi, lane) : te - tb;
+      if (lane == t) { ob = tb + a; oe = tb + b; }
+    }
+  } else if (lane < nops && windowed) {
     const int32_t* L = P.adj + ob;
     const int n = (int)(oe - ob);
     const int a = lo > 0 ? lower_bound_dev(L, n, lo) : 0;
@@ -151,8 +206,13 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   if (r >= 0) {
     rtable = c.tables + (size_t)(r - 2) * P.E;
     const long long rsize = __shfl_sync(FULL, c.lsize, r);
-    ra = lo > 0 ? paged_lower_bound(P, rtable, 0, rsize, lo) : 0;
-    rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
+    if (P.coop_window) {
+      ra = lo > 0 ? warp_paged_lower_bound(P, rtable, 0, rsize, lo, lane) : 0;
+      rb = hi < INT_MAX ? warp_paged_lower_bound(P, rtable, ra, rsize, hi, lane) : rsize;
+    } else {
+      ra = lo > 0 ? paged_lower_bound(P, rtable, 0, rsize, lo) : 0;
+      rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
+    }
     if (ra >= rb) return 0;
   }
   const uint32_t injm = pl.inj_mask[d];
@@ -176,7 +236,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       }
     }
     const long long total = len - __popc(__ballot_sync(FULL, hit));
-    if (STATS && lane == d) c.lnodes += (unsigned long long)total;
+    if (STATS && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
     return total;
   }
 
@@ -198,6 +258,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     const unsigned z = __ballot_sync(FULL, lane < nops && oe <= ob);
     if (z) return 0;
   }
+  if (MODE_OUT == 3 && eA - bA > (long long)P.fcap) return -2;
   const uint32_t others = __ballot_sync(FULL, lane < nops && lane != tA);
   const int need_label = (r >= 0 && pl.label[r] == pl.label[d]) ? -1 : pl.label[d];
   const int dmin = (r >= 0 && pl.deg_min[r] >= pl.deg_min[d]) ? 0 : pl.deg_min[d];
@@ -274,6 +335,8 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     const int cnt = __popc(bal);
     if (MODE_OUT == 0) {
       if (!paged_write(P, w, bal, total, v, lane)) return -1;
+    } else if (MODE_OUT == 3) {
+      if (ok) c.sF[total + __popc(bal & lanemask_lt())] = v;
     } else if (MODE_OUT == 2 && cnt) {
       unsigned long long ob0 = 0;
       if (lane == 0) ob0 = atomicAdd(ctr(P, C_OUTCUR), (unsigned long long)cnt);
@@ -288,7 +351,80 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     }
     total += cnt;
   }
-  if (STATS && lane == d) c.lnodes += (unsigned long long)total;
+  if (MODE_OUT == 3) __syncwarp();
+  if (STATS && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
+  return total;
+}
+
+// Leaf of a count job with the staged set F = sF[0, nF) (sorted, all S[k-2]-independent
+// filters applied): |F ∩ window(x) ∩ N(x)| when N(x) is an operand, else |F ∩ window(x)|
+// minus x itself, where x = S[k-2].  Either F is streamed
+// from shared memory and N(x) probed (hub bitmap, else per-lane binary search with an
+// advancing lower bound), or N(x) is streamed with coalesced loads -- first narrowed to
+// [F_min, F_max] by a warp-cooperative search -- and F probed in shared memory.
+template <bool STATS>
+__device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, int nF, int x) {
+  const DevPlan& pl = P.plan;
+  const int lane = c.lane;
+  const int* F = c.sF;
+  int lo = 0, hi = nF;
+  if (pl.lf_lo_var) lo = smem_lower_bound(F, 0, nF, x + 1);
+  if (pl.lf_hi_var) hi = smem_lower_bound(F, lo, nF, x);
+  if (lo >= hi) return 0;
+  if (!pl.lf_var) {
+    long long cnt = hi - lo;
+    if (pl.lf_inj_var) {
+      const int i = smem_lower_bound(F, lo, hi, x);
+      cnt -= (i < hi && F[i] == x) ? 1 : 0;
+    }
+    return cnt;
+  }
+  const long long b0 = __ldg(P.offs + x), b1 = __ldg(P.offs + x + 1);
+  const int hid = P.hub_id ? __ldg(P.hub_id + x) : -1;
+  const long long a = hi - lo, b = b1 - b0;
+  if (b == 0) return 0;
+  long long total = 0;
+  // cost model in "dependent global load" units: stream F and probe N(x) costs
+  // ceil(a/32) rounds of one binary search over N(x); streaming N(x) costs a window
+  // search plus ceil(b/32) rounds of one load and a shared-memory search over F
+  const int lgb = 32 - __clz((int)min(b, (long long)INT_MAX));
+  const int lga = 32 - __clz((int)a);
+  const long long costA = ((a + 31) >> 5) * (long long)(hid >= 0 ? P.lf_cost_g : lgb * P.lf_cost_g);
+  const long long costB = 3ll * P.lf_cost_g + ((b + 31) >> 5) * (long long)(P.lf_cost_g + lga);
+  if (costA <= costB) {
+    long long pb = b0;  // advancing lower bound into N(x)
+    for (int base = lo; base < hi; base += 32) {
+      const int i = base + lane;
+      const bool inr = i < hi;
+      const int v = inr ? F[i] : INT_MAX;
+      bool ok = inr;
+      if (hid >= 0) {
+        if (ok) ok = (__ldg(P.hub_bits + (long long)hid * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
+      } else {
+        const int last_lane = min(31, hi - 1 - base);
+        int pos = (int)(b1 - pb);
+        if (inr) pos = lower_bound_dev(P.adj + pb, (int)(b1 - pb), v);
+        ok = ok && pos < b1 - pb && __ldg(P.adj + pb + pos) == v;
+        pb += __shfl_sync(FULL, pos, last_lane);
+      }
+      total += __popc(__ballot_sync(FULL, ok));
+      if (hid < 0 && pb >= b1) break;
+    }
+  } else {
+    const int fmin = F[lo], fmax = F[hi - 1];
+    long long s = b0 + warp_lower_bound(P.adj + b0, b, fmin, lane);
+    for (; s < b1; s += 32) {
+      const long long i = s + lane;
+      const int v = i < b1 ? __ldg(P.adj + i) : INT_MAX;
+      bool ok = v <= fmax;
+      if (ok) {
+        const int j = smem_lower_bound(F, lo, hi, v);
+        ok = F[j] == v;  // j < hi since v <= fmax
+      }
+      total += __popc(__ballot_sync(FULL, ok));
+      if (__shfl_sync(FULL, v, 31) >= fmax) break;
+    }
+  }
   return total;
 }
 
@@ -324,10 +460,17 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
     c.count += (unsigned long long)n;
     return true;
   }
+  // leaf staging (count jobs): F of the virtual position kVF, once per level-(k-2) list
+  const bool use_lf = MODE == 0 && !STATS && P.plan.lf_on && P.fcap > 0;
+  int nF = -1;  // staged |F|, -1 = not staged (generic Eq. (1) per leaf)
   int d = start;
   long long sz = extend<0, STATS>(P, c, d, own2);
   if (sz < 0) return false;
   if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
+  if (use_lf && d == k - 2) {
+    nF = sz >= 2 ? (int)extend<3, STATS>(P, c, kVF, own2) : -1;
+    if (nF == 0 && lane == d) c.liter = (int)sz;  // F empty: no leaf below this list
+  }
   bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
   for (;;) {
     const int it = __shfl_sync(FULL, c.liter, d);
@@ -352,13 +495,19 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
       const int v = paged_read(P, table, it);
       if (lane == d) { c.sreg = v; c.liter = it + 1; }
       if (d + 1 == k - 1) {
-        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
+        long long n;
+        if (use_lf && nF >= 0) n = leaf_staged(P, c, nF, v);
+        else n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
         c.count += (unsigned long long)n;
       } else {
         d++;
         sz = extend<0, STATS>(P, c, d, own2);
         if (sz < 0) return false;
         if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
+        if (use_lf && d == k - 2) {
+          nF = sz >= 2 ? (int)extend<3, STATS>(P, c, kVF, own2) : -1;
+          if (nF == 0 && lane == d) c.liter = (int)sz;
+        }
       }
     } else {
       if (d == start) break;
@@ -458,6 +607,8 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.lnodes = 0;
   c.wbytes = c.sbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
+  extern __shared__ int smem_stage[];
+  c.sF = smem_stage + (threadIdx.x >> 5) * P.fcap;
   const Queue q = make_queue(P);
   int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
   unsigned long long* cursor = ctr(P, C_CURSOR);
@@ -592,10 +743,11 @@ int cuda_fail(cudaError_t e, const char* what) {
 }  // namespace
 
 // ------------------------------------------------------------------ host side
-int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int* out) {
+int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int* out) {
   (void)device;
   int nb = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, pick_kernel(enumerate ? 1 : 0, stats), wpb * 32, 0);
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, pick_kernel(enumerate ? 1 : 0, stats), wpb * 32,
+                                                                (size_t)wpb * fcap * sizeof(int));
   if (e != cudaSuccess) return cuda_fail(e, "occupancy");
   *out = std::max(1, nb);
   return TDFS_OK;
@@ -617,6 +769,9 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   if (e != cudaSuccess) return cuda_fail(e, "device attribute");
   L->wpb = o->warps_per_block > 0 ? o->warps_per_block : 4;
   if (L->wpb > 32) return fail(TDFS_E_INVALID_ARG, "opts.warps_per_block must be <= 32");
+  L->fcap = kLeafStage;
+  if (const char* e = getenv("TDFS_FCAP")) L->fcap = atoi(e);  // tuning knob (experiments)
+  if (L->fcap < 0 || L->fcap > 8192) return fail(TDFS_E_INVALID_ARG, "TDFS_FCAP must be in [0, 8192]");
   if (o->blocks > 0) {
     L->blocks = o->blocks;
   } else {
@@ -624,7 +779,7 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
     for (int m = 0; m < 2; m++)
       for (int s = 0; s < 2; s++) {
         int nb = 0;
-        int rc = blocks_per_sm(dev, L->wpb, s != 0, m != 0, &nb);
+        int rc = blocks_per_sm(dev, L->wpb, s != 0, m != 0, L->fcap, &nb);
         if (rc) return rc;
         mn = std::min(mn, nb);
       }
@@ -690,7 +845,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.n = g->n;
   P.plan = p->dev;
   if (o->flags & TDFS_RUN_NO_REUSE) {
-    for (int i = 0; i < kMaxK; i++) { P.plan.reuse[i] = -1; P.plan.shortcut[i] &= 2; }
+    for (int i = 0; i <= kVF; i++) { P.plan.reuse[i] = -1; P.plan.shortcut[i] &= 2; }
     P.plan.reuse_enabled = 0;
   }
   if (o->flags & TDFS_RUN_NO_SHORTCUT)
@@ -710,6 +865,11 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.page_shift = L.page_shift;
   P.E = L.E;
   P.tau_ns = o->tau_ns;
+  P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
+  P.lf_cost_g = 6;
+  P.coop_window = 1;
+  if (const char* e = getenv("TDFS_COOP")) P.coop_window = atoi(e);  // tuning knob (experiments)
+  if (const char* e = getenv("TDFS_LF_COST")) P.lf_cost_g = atoi(e);  // tuning knob (experiments)
   P.merge_ratio = kMergeRatio;
   if (const char* e = getenv("TDFS_MERGE_RATIO")) P.merge_ratio = atoi(e);  // tuning knob (experiments)
   P.bsearch_variant = 0;
@@ -746,7 +906,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     cudaEventRecord(ev0, st);
   }
   KernelFn fn = pick_kernel(mode, want_stats);
-  fn<<<L.blocks, L.wpb * 32, 0, st>>>(P);
+  fn<<<L.blocks, L.wpb * 32, (size_t)L.wpb * L.fcap * sizeof(int), st>>>(P);
   if ((e = cudaGetLastError()) != cudaSuccess) {
     cudaFree(d_trace);
     return cuda_fail(e, "kernel launch");

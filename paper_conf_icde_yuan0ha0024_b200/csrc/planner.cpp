@@ -163,6 +163,38 @@ void build_dev(const QueryAdj& q, Plan& P) {
         d.shortcut[p] |= 1;
     }
   }
+  // Leaf staging: the virtual position kVF holds the S[k-2]-independent part of the last
+  // position (internal.h).  A superset start C(r) for it follows the reuse rule above with
+  // r <= k-2 (all stored lists of the current prefix are alive while level k-2 iterates).
+  d.lf_on = 0;
+  d.reuse[kVF] = -1;
+  d.shortcut[kVF] = 0;
+  if (q.k >= 4) {
+    const int p = q.k - 1, v = q.k - 2;
+    const uint32_t fixm = (1u << v) - 1u;
+    d.bwd[kVF] = d.bwd[p] & fixm;
+    d.lo_mask[kVF] = d.lo_mask[p] & fixm;
+    d.hi_mask[kVF] = d.hi_mask[p] & fixm;
+    d.inj_mask[kVF] = d.inj_mask[p] & fixm;
+    d.label[kVF] = d.label[p];
+    d.deg_min[kVF] = d.deg_min[p];
+    d.lf_var = (int8_t)((d.bwd[p] >> v) & 1u);
+    d.lf_lo_var = (int8_t)((d.lo_mask[p] >> v) & 1u);
+    d.lf_hi_var = (int8_t)((d.hi_mask[p] >> v) & 1u);
+    d.lf_inj_var = (int8_t)((d.inj_mask[p] >> v) & 1u);
+    d.lf_on = d.bwd[kVF] != 0;
+    int best = -1;
+    const int nb = __builtin_popcount(d.bwd[p]);
+    for (int r = 2; r <= v; r++) {
+      if ((d.bwd[r] & d.bwd[kVF]) != d.bwd[r]) continue;
+      if (d.label[r] >= 0 && d.label[r] != d.label[p]) continue;
+      if (d.deg_min[r] > std::max(d.deg_min[p], nb)) continue;
+      if ((d.lo_mask[r] & d.lo_mask[kVF]) != d.lo_mask[r]) continue;
+      if ((d.hi_mask[r] & d.hi_mask[kVF]) != d.hi_mask[r]) continue;
+      if (best < 0 || __builtin_popcount(d.bwd[r]) >= __builtin_popcount(d.bwd[best])) best = r;
+    }
+    d.reuse[kVF] = (int8_t)best;
+  }
   d.reuse_enabled = 1;
 }
 
