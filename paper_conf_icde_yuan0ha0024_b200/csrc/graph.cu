@@ -173,17 +173,14 @@ __global__ void hub_bits_kernel(const int64_t* __restrict__ offs, const int32_t*
 // Hub adjacency bitmaps: the highest-degree vertices (degree >= 256,
 // at most `budget` bytes of bitmaps) get an n-bit membership bitmap so that probing
 // w in N(hub) during Eq. (1) is one load instead of a binary search over a long list.
-int build_hub_bitmaps(Graph& G, cudaStream_t st) {
+int build_hub_bitmaps(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs, std::vector<int32_t>& hub_vertices) {
   const long long words = (G.n + 31) / 32;
   if (G.n == 0 || words == 0) return TDFS_OK;
   long long budget = 64ll << 20;
   if (const char* e = getenv("TDFS_HUB_BUDGET_MB")) budget = atoll(e) << 20;
   const long long max_hubs = budget / (words * 4);
   if (max_hubs <= 0) return TDFS_OK;
-  std::vector<int64_t> offs((size_t)G.n + 1);
-  cudaError_t e = cudaMemcpyAsync(offs.data(), G.d_offs, sizeof(int64_t) * (G.n + 1), cudaMemcpyDeviceToHost, st);
-  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  if (e != cudaSuccess) return cuda_fail(e, "hubs: offs copy");
+  cudaError_t e;
   std::vector<std::pair<int64_t, int32_t>> cand;
   const int64_t min_deg = 256;
   for (int64_t v = 0; v < G.n; v++) {
@@ -219,7 +216,78 @@ int build_hub_bitmaps(Graph& G, cudaStream_t st) {
   e = cudaStreamSynchronize(st);
   cudaFree(d_vert);
   if (e != cudaSuccess) return cuda_fail(e, "hubs: build");
+  hub_vertices = hub_vertex;
   return TDFS_OK;
+}
+
+// Per-vertex open-addressing hash sets of the adjacency lists:
+// vertex v with deg(v) >= kHashMinDeg owns T_v = next_pow2(2 deg(v)) int32 slots
+// (load factor <= 1/2) at hoff[v]; w sits at or after slot fib(w) >> (32 - log2 T_v),
+// linear probing, EMPTY = -1.  Membership w in N(v) during Eq. (1) then costs one
+// aligned 16-byte group load (rarely two) instead of log2 deg(v) dependent loads.
+// The sorted CSR stays the primary copy (streamed operands, windows, merge).
+__global__ void hash_fill_kernel(const int64_t* __restrict__ offs, const int32_t* __restrict__ adj, int64_t n,
+                                 const int64_t* __restrict__ hoff, int32_t* __restrict__ slots) {
+  const int64_t nwarps = (int64_t)gridDim.x * blockDim.x / 32;
+  const int lane = threadIdx.x & 31;
+  for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; v < n; v += nwarps) {
+    const int64_t h0 = hoff[v], T = hoff[v + 1] - h0;
+    if (T == 0) continue;
+    const int sh = 32 - (31 - __clz((int)T));  // 32 - log2 T
+    for (int64_t e = offs[v] + lane; e < offs[v + 1]; e += 32) {
+      const int32_t w = adj[e];
+      uint32_t s = ((uint32_t)w * 2654435769u) >> sh;
+      for (;;) {
+        const int old = atomicCAS(slots + h0 + s, -1, w);
+        if (old == -1 || old == w) break;
+        s = (s + 1) & (uint32_t)(T - 1);
+      }
+    }
+  }
+}
+
+int build_hash_index(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs,
+                     const std::vector<int32_t>& hub_vertices) {
+  G.hash_min_deg = kHashMinDeg;
+  if (const char* e = getenv("TDFS_HASH_MIN_DEG")) G.hash_min_deg = atoll(e);  // tuning knob (experiments)
+  if (G.n == 0 || G.hash_min_deg <= 0) return TDFS_OK;
+  // hubs are probed through their bitmaps everywhere, so they get no hash set
+  std::vector<char> is_hub((size_t)G.n, 0);
+  for (int32_t v : hub_vertices) is_hub[v] = 1;
+  std::vector<int64_t> hoff((size_t)G.n + 1, 0);
+  for (int64_t v = 0; v < G.n; v++) {
+    const int64_t d = offs[v + 1] - offs[v];
+    int64_t T = 0;
+    if (d >= G.hash_min_deg && !is_hub[v]) {
+      T = 4;
+      while (T < 2 * d) T <<= 1;
+    }
+    hoff[v + 1] = hoff[v] + T;
+  }
+  if (hoff[G.n] == 0) return TDFS_OK;
+  cudaError_t e;
+  if ((e = cudaMalloc(&G.d_hoff, sizeof(int64_t) * (G.n + 1))) != cudaSuccess ||
+      (e = cudaMalloc(&G.d_hslots, sizeof(int32_t) * (size_t)hoff[G.n])) != cudaSuccess)
+    return fail(TDFS_E_OOM, "hash index: alloc");
+  G.hash_slots = hoff[G.n];
+  cudaMemcpyAsync(G.d_hoff, hoff.data(), sizeof(int64_t) * (G.n + 1), cudaMemcpyHostToDevice, st);
+  cudaMemsetAsync(G.d_hslots, 0xff, sizeof(int32_t) * (size_t)hoff[G.n], st);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, G.device);
+  hash_fill_kernel<<<sms * 8, 256, 0, st>>>(G.d_offs, G.d_adj, G.n, G.d_hoff, G.d_hslots);
+  if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "hash index: build");
+  return TDFS_OK;
+}
+
+int build_indexes(Graph& G, cudaStream_t st) {
+  std::vector<int64_t> offs((size_t)G.n + 1);
+  cudaError_t e = cudaMemcpyAsync(offs.data(), G.d_offs, sizeof(int64_t) * (G.n + 1), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(e, "index: offs copy");
+  std::vector<int32_t> hubs;
+  int rc = build_hub_bitmaps(G, st, offs, hubs);
+  if (rc == TDFS_OK) rc = build_hash_index(G, st, offs, hubs);
+  return rc;
 }
 
 int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enforce = false) {
@@ -246,7 +314,7 @@ int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enf
     G.nlabels = G.d_label ? (int32_t)h[2] + 1 : 1;
   }
   if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "load: sync");
-  return build_hub_bitmaps(G, st);
+  return build_indexes(G, st);
 }
 
 void release(Graph& G) {
@@ -258,6 +326,9 @@ void release(Graph& G) {
   cudaFree(G.d_src);
   cudaFree(G.d_hub_id);
   cudaFree(G.d_hub_bits);
+  cudaFree(G.d_hoff);
+  cudaFree(G.d_hslots);
+  G.d_hoff = nullptr; G.d_hslots = nullptr; G.hash_slots = 0;
   G.d_offs = nullptr; G.d_adj = nullptr; G.d_label = nullptr; G.d_src = nullptr;
   G.d_hub_id = nullptr; G.d_hub_bits = nullptr; G.n_hubs = 0;
 }

@@ -28,7 +28,8 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // list and staged in shared memory; each leaf is then
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
-constexpr int kLeafStage = 512;  // default shared-memory ids per warp for the leaf set F
+constexpr int kLeafStage = 512;
+constexpr int64_t kHashMinDeg = 32;  // lists shorter than this are searched (they span <= 2 cache lines)  // default shared-memory ids per warp for the leaf set F
 struct DevPlan {
   int32_t k;
   int32_t order[kMaxK];          // query vertex at position p (enumerate output mapping)
@@ -47,6 +48,7 @@ struct DevPlan {
   int8_t lf_var;                 // N(S[k-2]) is an operand of position k-1
   int8_t lf_lo_var, lf_hi_var;   // window bound v > S[k-2] / v < S[k-2]
   int8_t lf_inj_var;             // v != S[k-2] must be tested (not implied)
+  int8_t lf_byref;               // F = a window of one adjacency list, no per-element filter (FRef by reference)
 };
 
 struct Plan {
@@ -73,6 +75,10 @@ struct Graph {
   int32_t* d_hub_id = nullptr;     // [n], -1 for non-hubs
   uint32_t* d_hub_bits = nullptr;  // [n_hubs][hub_words]
   int64_t n_hubs = 0, hub_words = 0, hub_min_deg = 0;
+  // per-vertex adjacency hash sets (deg >= hash_min_deg), DESIGN.md "hash index"
+  int64_t* d_hoff = nullptr;       // [n+1] slot offsets, T_v = hoff[v+1]-hoff[v] (0 or a power of two)
+  int32_t* d_hslots = nullptr;     // EMPTY = -1
+  int64_t hash_slots = 0, hash_min_deg = 0;
 };
 
 // ---------------------------------------------------------------- device job
@@ -109,7 +115,8 @@ struct KParams {
   int32_t n_levels;            // stored stack levels = max(0, k - 3): positions 2 .. k-2
   // queue
   QSlot* slots;
-  uint64_t qcap;
+  uint64_t qcap;                // capacity in tasks (initial value of the `free` counter)
+  uint64_t qslots;              // ring slots: next power of two >= qcap (index = ticket & (qslots - 1))
   // counters
   unsigned long long* ctr;     // C_NUM * kCounterStride u64
   unsigned long long* stats;   // S_NUM u64 or nullptr
@@ -121,14 +128,20 @@ struct KParams {
   int32_t E;                   // page-table entries per level
   int64_t tau_ns;              // < 0: infinity
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
+  int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
-  int32_t lf_cost_g;           // leaf staging cost model: one dependent global load in shared-memory steps
+  int32_t lf_byref;            // leaf staging: reference F in place when the plan allows (else materialise)
+  int32_t lf_cost_g;
+  int32_t lf_cost_h;           // leaf staging cost model: extra cost of a hash probe over a bitmap probe           // leaf staging cost model: one dependent global load in shared-memory steps
   int32_t coop_window;         // constraint windows by warp-cooperative 32-ary search (else per-lane binary)
   int32_t bsearch_variant;     // 0 halving, 1 power-of-two (experiments)
   // hub bitmaps (nullptr when off)
   const int32_t* hub_id;
   const uint32_t* hub_bits;
   long long hub_words;
+  // adjacency hash sets (nullptr when off)
+  const int64_t* hoff;
+  const int32_t* hslots;
   // enumerate
   int32_t* out;
   unsigned long long cap;
@@ -140,7 +153,7 @@ struct KParams {
 // workspace layout (byte offsets from the 256-aligned base)
 struct WsLayout {
   size_t ctr = 0, stats = 0, slots = 0, tables = 0, pool = 0, total = 0;
-  uint64_t qcap = 0, n_pages = 0;
+  uint64_t qcap = 0, qslots = 0, n_pages = 0;
   int32_t E = 0, page_shift = 0, n_levels = 0, blocks = 0, wpb = 0, fcap = 0;
 };
 

@@ -151,10 +151,16 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   const int sj = __shfl_sync(FULL, c.sreg, jt);
   long long ob = 0, oe = 0;
   int hid = -1;
+  long long hb = 0;  // hash set of the operand: slots [hb, hb + hT), hT = 0 if none
+  unsigned hT = 0;
   if (lane < nops) {
     ob = __ldg(P.offs + sj);
     oe = __ldg(P.offs + sj + 1);
     if (P.hub_id) hid = __ldg(P.hub_id + sj);
+    if (P.hoff) {
+      hb = __ldg(P.hoff + sj);
+      hT = (unsigned)(__ldg(P.hoff + sj + 1) - hb);
+    }
   }
   if (STATS && MODE_OUT != 3) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
     const bool mine = (bm_all >> lane) & 1u;
@@ -206,13 +212,19 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   if (r >= 0) {
     rtable = c.tables + (size_t)(r - 2) * P.E;
     const long long rsize = __shfl_sync(FULL, c.lsize, r);
-    if (P.coop_window) {
-      ra = lo > 0 ? warp_paged_lower_bound(P, rtable, 0, rsize, lo, lane) : 0;
-      rb = hi < INT_MAX ? warp_paged_lower_bound(P, rtable, ra, rsize, hi, lane) : rsize;
-    } else {
-      ra = lo > 0 ? paged_lower_bound(P, rtable, 0, rsize, lo) : 0;
-      rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
+    // when the window includes v > S[r]: C(r) is sorted and S[r] = C(r)[iter[r] - 1], so the
+    // window starts at or after iter[r] -- exactly there when lo = S[r] + 1 (no search)
+    long long r0 = 0;
+    bool ra_known = false;
+    if ((lom >> r) & 1u) {
+      r0 = __shfl_sync(FULL, c.liter, r);
+      ra_known = (lo == getS(c.sreg, r) + 1);
     }
+    if (ra_known) ra = r0;
+    else if (P.coop_window) ra = lo > 0 ? warp_paged_lower_bound(P, rtable, r0, rsize, lo, lane) : 0;
+    else ra = lo > 0 ? paged_lower_bound(P, rtable, r0, rsize, lo) : 0;
+    if (P.coop_window) rb = hi < INT_MAX ? warp_paged_lower_bound(P, rtable, ra, rsize, hi, lane) : rsize;
+    else rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
     if (ra >= rb) return 0;
   }
   const uint32_t injm = pl.inj_mask[d];
@@ -289,7 +301,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       if (th >= 0) {
         // hub operand: one bitmap load per candidate (v is inside the window already)
         if (ok) ok = (__ldg(P.hub_bits + (long long)th * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
-      } else if ((te - tb) <= (long long)P.merge_ratio * (eA - base)) {
+      } else if ((te - tb) <= (long long)(__shfl_sync(FULL, hT, t) ? P.merge_ratio_hash : P.merge_ratio) * (eA - base)) {
         // warp merge: walk B in coalesced 32-id chunks until a chunk reaches the batch max
         const int amax = __shfl_sync(FULL, v, last_lane);
         bool found = false;
@@ -308,6 +320,10 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
         }
         ok = ok && found;
         if (lane == t) ob = min(ptr, te);
+      } else if (const unsigned tT = __shfl_sync(FULL, hT, t)) {
+        // hashed operand: one aligned 16-byte group load per candidate (rarely two)
+        const long long th0 = __shfl_sync(FULL, hb, t);
+        if (ok) ok = hash_contains(P.hslots, th0, tT, v);
       } else {
         int pos = (int)(te - tb);
         const bool probe = inr && (ok || lane == last_lane);
@@ -362,70 +378,194 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
 // from shared memory and N(x) probed (hub bitmap, else per-lane binary search with an
 // advancing lower bound), or N(x) is streamed with coalesced loads -- first narrowed to
 // [F_min, F_max] by a warp-cooperative search -- and F probed in shared memory.
+// Per-vertex probe metadata of N(x): CSR range, hub bitmap row, hash set.
+struct VMeta {
+  long long b0, b1;  // N(x) = adj[b0, b1)
+  long long hb;      // hash slots [hb, hb + hT)
+  unsigned hT;       // 0 = no hash set
+  int hid;           // hub bitmap row, -1 = none
+};
+
+__device__ __forceinline__ VMeta load_vmeta(const KParams& P, int x) {
+  VMeta m;
+  m.b0 = __ldg(P.offs + x);
+  m.b1 = __ldg(P.offs + x + 1);
+  m.hid = P.hub_id ? __ldg(P.hub_id + x) : -1;
+  m.hb = 0;
+  m.hT = 0;
+  if (P.hoff) {
+    m.hb = __ldg(P.hoff + x);
+    m.hT = (unsigned)(__ldg(P.hoff + x + 1) - m.hb);
+  }
+  return m;
+}
+
+__device__ __forceinline__ VMeta shfl_vmeta(const VMeta& m, int src) {
+  VMeta r;
+  r.b0 = __shfl_sync(FULL, m.b0, src);
+  r.b1 = __shfl_sync(FULL, m.b1, src);
+  r.hb = __shfl_sync(FULL, m.hb, src);
+  r.hT = __shfl_sync(FULL, m.hT, src);
+  r.hid = __shfl_sync(FULL, m.hid, src);
+  return r;
+}
+
+// The staged leaf set F of a level-(k-2) list: either materialised in this warp's shared
+// memory (sorted, every S[k-2]-independent filter applied), or -- when F is a window of a
+// single adjacency list N(y) with no per-element filter (lf_byref) and y has a bitmap or
+// hash set -- referenced in place: F = adj[offs[y] + a, offs[y] + b) and "w in F" is
+// "w in [F_min, F_max] and w in N(y)" by y's bitmap / hash set (no copy, no size cap).
+struct FRef {
+  const int* F;  // sorted ids F[0, nF) (shared or global memory)
+  int hid;       // by reference: y's bitmap row, -1 = none
+  long long hb;  // by reference: y's hash set slots [hb, hb + hT)
+  unsigned hT;   // 0 = none; hid < 0 && hT == 0 means F is materialised in shared memory
+};
+
+// |{ v in L[s, e) : vmin <= v <= vmax, v in set }| for a sorted list L (global or shared
+// memory) and an O(1) probe set (bitmap row, else hash set).  Two 32-id batches per
+// round so that two probe loads per lane are in flight; stops past vmax.
+__device__ long long count_stream_probe(const KParams& P, const int* L, long long s, long long e, int vmin, int vmax,
+                                        int hid, long long hb, unsigned hT, int lane) {
+  const uint32_t* row = hid >= 0 ? P.hub_bits + (long long)hid * P.hub_words : nullptr;
+  long long total = 0;
+  for (long long base = s; base < e; base += 64) {
+    const long long i0 = base + lane, i1 = i0 + 32;
+    const int v0 = i0 < e ? L[i0] : INT_MAX, v1 = i1 < e ? L[i1] : INT_MAX;
+    const bool in0 = i0 < e && v0 >= vmin && v0 <= vmax;
+    const bool in1 = i1 < e && v1 >= vmin && v1 <= vmax;
+    bool ok0, ok1;
+    if (row) {
+      const uint32_t w0 = in0 ? __ldg(row + (v0 >> 5)) : 0u;
+      const uint32_t w1 = in1 ? __ldg(row + (v1 >> 5)) : 0u;
+      ok0 = (w0 >> (v0 & 31)) & 1u;
+      ok1 = (w1 >> (v1 & 31)) & 1u;
+    } else {
+      const unsigned s0 = hash_home(hT, v0), s1 = hash_home(hT, v1);
+      const int4 q0 = in0 ? __ldg(reinterpret_cast<const int4*>(P.hslots + hb + (s0 & ~3u))) : make_int4(0, 0, 0, -1);
+      const int4 q1 = in1 ? __ldg(reinterpret_cast<const int4*>(P.hslots + hb + (s1 & ~3u))) : make_int4(0, 0, 0, -1);
+      int r0 = in0 ? hash_group(q0, v0, s0 & 3u) : 0;
+      int r1 = in1 ? hash_group(q1, v1, s1 & 3u) : 0;
+      if (r0 < 0) r0 = hash_tail(P.hslots, hb, hT, v0, s0 & ~3u);
+      if (r1 < 0) r1 = hash_tail(P.hslots, hb, hT, v1, s1 & ~3u);
+      ok0 = r0 > 0;
+      ok1 = r1 > 0;
+    }
+    total += __popc(__ballot_sync(FULL, ok0)) + __popc(__ballot_sync(FULL, ok1));
+    if (__any_sync(FULL, (i1 < e ? v1 : (i0 < e ? v0 : INT_MIN)) > vmax)) break;
+  }
+  return total;
+}
+
+// lower_bound of v in F[lo, hi): shared-memory halving search, or a warp-cooperative
+// 32-ary search when F is referenced in global memory
+__device__ __forceinline__ int f_lower_bound(const FRef& fr, int lo, int hi, int v, int lane) {
+  if (fr.hid >= 0 || fr.hT) return lo + (int)warp_lower_bound(fr.F + lo, hi - lo, v, lane);
+  return smem_lower_bound(fr.F, lo, hi, v);
+}
+
+// Leaf of a count job with the staged set F[0, nF) (fr): |F ∩ window(x) ∩ N(x)| when N(x)
+// is an operand, else |F ∩ window(x)| minus x itself, where x = S[k-2] (DESIGN.md "leaf
+// staging"); mx = N(x)'s metadata (loaded in batches of 32 leaves by the caller).  A cost
+// model picks one of: stream F and probe N(x) (hub bitmap, else hash set, else per-lane
+// binary search with an advancing lower bound), or stream N(x) -- narrowed to
+// [F_min, F_max] by a warp-cooperative search -- and probe F (y's bitmap / hash set when
+// F is referenced, else a shared-memory binary search).
 template <bool STATS>
-__device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, int nF, int x) {
+__device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, const FRef& fr, int nF, int x, const VMeta& mx) {
   const DevPlan& pl = P.plan;
   const int lane = c.lane;
-  const int* F = c.sF;
+  const int* F = fr.F;
+  const bool byref = fr.hid >= 0 || fr.hT;
   int lo = 0, hi = nF;
-  if (pl.lf_lo_var) lo = smem_lower_bound(F, 0, nF, x + 1);
-  if (pl.lf_hi_var) hi = smem_lower_bound(F, lo, nF, x);
+  if (pl.lf_lo_var) lo = f_lower_bound(fr, 0, nF, x + 1, lane);
+  if (pl.lf_hi_var) hi = f_lower_bound(fr, lo, nF, x, lane);
   if (lo >= hi) return 0;
   if (!pl.lf_var) {
     long long cnt = hi - lo;
     if (pl.lf_inj_var) {
-      const int i = smem_lower_bound(F, lo, hi, x);
+      const int i = f_lower_bound(fr, lo, hi, x, lane);
       cnt -= (i < hi && F[i] == x) ? 1 : 0;
     }
     return cnt;
   }
-  const long long b0 = __ldg(P.offs + x), b1 = __ldg(P.offs + x + 1);
-  const int hid = P.hub_id ? __ldg(P.hub_id + x) : -1;
+  const long long b0 = mx.b0, b1 = mx.b1;
+  const int hid = mx.hid;
+  const unsigned hT = mx.hT;
   const long long a = hi - lo, b = b1 - b0;
   if (b == 0) return 0;
-  long long total = 0;
   // cost model in "dependent global load" units: stream F and probe N(x) costs
-  // ceil(a/32) rounds of one binary search over N(x); streaming N(x) costs a window
-  // search plus ceil(b/32) rounds of one load and a shared-memory search over F
+  // ceil(a/32) rounds of one probe of N(x); streaming N(x) costs a window
+  // search plus ceil(b/32) rounds of one load and one probe of F
+  const int g = P.lf_cost_g;
   const int lgb = 32 - __clz((int)min(b, (long long)INT_MAX));
   const int lga = 32 - __clz((int)a);
-  const long long costA = ((a + 31) >> 5) * (long long)(hid >= 0 ? P.lf_cost_g : lgb * P.lf_cost_g);
-  const long long costB = 3ll * P.lf_cost_g + ((b + 31) >> 5) * (long long)(P.lf_cost_g + lga);
+  const long long costA = ((a + 31) >> 5) * (long long)(hid >= 0 ? g : hT ? g + P.lf_cost_h : lgb * g);
+  const long long costB = 3ll * g + ((b + 31) >> 5) * (long long)(byref ? 2 * g + P.lf_cost_h : g + lga);
+  if (costA <= costB && (hid >= 0 || hT)) return count_stream_probe(P, F, lo, hi, INT_MIN, INT_MAX, hid, mx.hb, hT, lane);
+  long long total = 0;
   if (costA <= costB) {
     long long pb = b0;  // advancing lower bound into N(x)
     for (int base = lo; base < hi; base += 32) {
       const int i = base + lane;
       const bool inr = i < hi;
       const int v = inr ? F[i] : INT_MAX;
-      bool ok = inr;
-      if (hid >= 0) {
-        if (ok) ok = (__ldg(P.hub_bits + (long long)hid * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
-      } else {
-        const int last_lane = min(31, hi - 1 - base);
-        int pos = (int)(b1 - pb);
-        if (inr) pos = lower_bound_dev(P.adj + pb, (int)(b1 - pb), v);
-        ok = ok && pos < b1 - pb && __ldg(P.adj + pb + pos) == v;
-        pb += __shfl_sync(FULL, pos, last_lane);
-      }
+      const int last_lane = min(31, hi - 1 - base);
+      int pos = (int)(b1 - pb);
+      if (inr) pos = lower_bound_dev(P.adj + pb, (int)(b1 - pb), v);
+      const bool ok = inr && pos < b1 - pb && __ldg(P.adj + pb + pos) == v;
+      pb += __shfl_sync(FULL, pos, last_lane);
       total += __popc(__ballot_sync(FULL, ok));
-      if (hid < 0 && pb >= b1) break;
+      if (pb >= b1) break;
     }
-  } else {
-    const int fmin = F[lo], fmax = F[hi - 1];
-    long long s = b0 + warp_lower_bound(P.adj + b0, b, fmin, lane);
-    for (; s < b1; s += 32) {
-      const long long i = s + lane;
-      const int v = i < b1 ? __ldg(P.adj + i) : INT_MAX;
-      bool ok = v <= fmax;
-      if (ok) {
-        const int j = smem_lower_bound(F, lo, hi, v);
-        ok = F[j] == v;  // j < hi since v <= fmax
-      }
-      total += __popc(__ballot_sync(FULL, ok));
-      if (__shfl_sync(FULL, v, 31) >= fmax) break;
+    return total;
+  }
+  const int fmin = F[lo], fmax = F[hi - 1];
+  const long long s = b0 + (b > 64 ? warp_lower_bound(P.adj + b0, b, fmin, lane) : 0);
+  if (byref) return count_stream_probe(P, P.adj, s, b1, fmin, fmax, fr.hid, fr.hb, fr.hT, lane);
+  for (long long sb = s; sb < b1; sb += 32) {
+    const long long i = sb + lane;
+    const int v = i < b1 ? __ldg(P.adj + i) : INT_MAX;
+    bool ok = v >= fmin && v <= fmax;
+    if (ok) {
+      const int j = smem_lower_bound(F, lo, hi, v);
+      ok = F[j] == v;  // j < hi since v <= fmax
     }
+    total += __popc(__ballot_sync(FULL, ok));
+    if (__shfl_sync(FULL, v, 31) >= fmax) break;
   }
   return total;
+}
+
+// Stage F for the level-(k-2) list just built (see FRef).  Returns |F|, or -2 when F
+// would have to be materialised and exceeds the shared-memory stage (generic per leaf).
+template <bool STATS>
+__device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& fr) {
+  const DevPlan& pl = P.plan;
+  const int lane = c.lane;
+  fr.F = c.sF;
+  fr.hid = -1;
+  fr.hb = 0;
+  fr.hT = 0;
+  if (pl.lf_byref && P.lf_byref) {
+    const int y = getS(c.sreg, __ffs(pl.bwd[kVF]) - 1);
+    const VMeta my = load_vmeta(P, y);
+    if (my.hid >= 0 || my.hT) {
+      const uint32_t lom = pl.lo_mask[kVF], him = pl.hi_mask[kVF];
+      const int wlo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
+      const int whi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
+      if (wlo >= whi) return 0;
+      const long long n = my.b1 - my.b0;
+      const long long a = wlo > 0 ? warp_lower_bound(P.adj + my.b0, n, wlo, lane) : 0;
+      const long long b = whi < INT_MAX ? a + warp_lower_bound(P.adj + my.b0 + a, n - a, whi, lane) : n;
+      fr.F = P.adj + my.b0 + a;
+      fr.hid = my.hid;
+      fr.hb = my.hb;
+      fr.hT = my.hT;
+      return (int)(b - a);
+    }
+  }
+  return (int)extend<3, STATS>(P, c, kVF, own2);
 }
 
 // Push <S0, S1, L[2][i]> for i in [from, size) -- timeout split of level 2
@@ -463,12 +603,13 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
   // leaf staging (count jobs): F of the virtual position kVF, once per level-(k-2) list
   const bool use_lf = MODE == 0 && !STATS && P.plan.lf_on && P.fcap > 0;
   int nF = -1;  // staged |F|, -1 = not staged (generic Eq. (1) per leaf)
+  FRef fr;
   int d = start;
   long long sz = extend<0, STATS>(P, c, d, own2);
   if (sz < 0) return false;
   if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
   if (use_lf && d == k - 2) {
-    nF = sz >= 2 ? (int)extend<3, STATS>(P, c, kVF, own2) : -1;
+    nF = sz >= 2 ? stage_leaf_set(P, c, own2, fr) : -1;
     if (nF == 0 && lane == d) c.liter = (int)sz;  // F empty: no leaf below this list
   }
   bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
@@ -492,12 +633,23 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
       }
       if (d == 2) grace = false;
       const uint32_t* table = c.tables + (size_t)(d - 2) * P.E;
+      if (d + 1 == k - 1 && use_lf && nF >= 0) {
+        // staged leaves in batches of 32: the ids and N(x) metadata of the batch are
+        // loaded by one lane each (independent loads), then each leaf is one |F ∩ N(x)|
+        const int nb = min(32, size - it);
+        const int vl = lane < nb ? paged_read(P, table, it + lane) : 0;
+        VMeta ml;
+        if (lane < nb) ml = load_vmeta(P, vl);
+        long long n = 0;
+        for (int j = 0; j < nb; j++) n += leaf_staged(P, c, fr, nF, __shfl_sync(FULL, vl, j), shfl_vmeta(ml, j));
+        c.count += (unsigned long long)n;
+        if (lane == d) c.liter = it + nb;
+        continue;
+      }
       const int v = paged_read(P, table, it);
       if (lane == d) { c.sreg = v; c.liter = it + 1; }
       if (d + 1 == k - 1) {
-        long long n;
-        if (use_lf && nF >= 0) n = leaf_staged(P, c, nF, v);
-        else n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
+        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
         c.count += (unsigned long long)n;
       } else {
         d++;
@@ -505,7 +657,7 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         if (sz < 0) return false;
         if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
         if (use_lf && d == k - 2) {
-          nF = sz >= 2 ? (int)extend<3, STATS>(P, c, kVF, own2) : -1;
+          nF = sz >= 2 ? stage_leaf_set(P, c, own2, fr) : -1;
           if (nF == 0 && lane == d) c.liter = (int)sz;
         }
       }
@@ -795,6 +947,8 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   long long need = std::max<long long>(1, (g->dmax + ints_per_page - 1) / ints_per_page);
   L->E = o->page_table_entries > 0 ? o->page_table_entries : (int)need;
   L->qcap = (uint64_t)(o->queue_ints / 3);
+  L->qslots = 1;
+  while (L->qslots < L->qcap) L->qslots <<= 1;
   if (o->pool_bytes > 0) {
     L->n_pages = (uint64_t)(o->pool_bytes / o->page_bytes);
   } else {
@@ -813,7 +967,7 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   L->stats = off;
   off += align_up(sizeof(unsigned long long) * S_NUM, 256);
   L->slots = off;
-  off += align_up(sizeof(QSlot) * L->qcap, 256);
+  off += align_up(sizeof(QSlot) * L->qslots, 256);
   L->tables = off;
   off += align_up(sizeof(uint32_t) * (size_t)n_warps * std::max(L->n_levels, 1) * L->E, 256);
   L->pool = off;
@@ -857,6 +1011,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.n_levels = L.n_levels;
   P.slots = (QSlot*)(base + L.slots);
   P.qcap = L.qcap;
+  P.qslots = L.qslots;
   P.ctr = (unsigned long long*)(base + L.ctr);
   P.stats = want_stats ? (unsigned long long*)(base + L.stats) : nullptr;
   P.page_tables = (uint32_t*)(base + L.tables);
@@ -867,16 +1022,26 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
   P.lf_cost_g = 6;
+  P.lf_cost_h = 2;
+  if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
+  P.lf_byref = 1;
+  if (const char* e = getenv("TDFS_BYREF")) P.lf_byref = atoi(e);  // tuning knob (experiments)
   P.coop_window = 1;
   if (const char* e = getenv("TDFS_COOP")) P.coop_window = atoi(e);  // tuning knob (experiments)
   if (const char* e = getenv("TDFS_LF_COST")) P.lf_cost_g = atoi(e);  // tuning knob (experiments)
   P.merge_ratio = kMergeRatio;
   if (const char* e = getenv("TDFS_MERGE_RATIO")) P.merge_ratio = atoi(e);  // tuning knob (experiments)
+  P.merge_ratio_hash = kMergeRatioHash;
+  if (const char* e = getenv("TDFS_MERGE_RATIO_H")) P.merge_ratio_hash = atoi(e);  // tuning knob (experiments)
   P.bsearch_variant = 0;
   if (g->d_hub_bits && !(o->flags & TDFS_RUN_NO_HUB_BITMAP)) {
     P.hub_id = g->d_hub_id;
     P.hub_bits = g->d_hub_bits;
     P.hub_words = g->hub_words;
+  }
+  if (g->d_hslots && !(o->flags & TDFS_RUN_NO_HASH)) {
+    P.hoff = g->d_hoff;
+    P.hslots = g->d_hslots;
   }
   if (const char* e = getenv("TDFS_BSEARCH")) P.bsearch_variant = atoi(e);
   P.out = d_out;
@@ -893,8 +1058,8 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   init_counters_kernel<<<1, C_NUM * kCounterStride, 0, st>>>(P.ctr, P.qcap, ticket_base);
   if (want_stats) cudaMemsetAsync(P.stats, 0, sizeof(unsigned long long) * S_NUM, st);
   {
-    int nb = (int)std::min<uint64_t>((L.qcap + 255) / 256, 4096);
-    init_queue_kernel<<<std::max(nb, 1), 256, 0, st>>>(P.slots, P.qcap, ticket_base);
+    int nb = (int)std::min<uint64_t>((L.qslots + 255) / 256, 4096);
+    init_queue_kernel<<<std::max(nb, 1), 256, 0, st>>>(P.slots, P.qslots, ticket_base);
   }
   size_t tbytes = sizeof(uint32_t) * (size_t)L.blocks * L.wpb * std::max(L.n_levels, 1) * L.E;
   if (L.n_levels > 0) cudaMemsetAsync(P.page_tables, 0xff, tbytes, st);

@@ -5,6 +5,7 @@
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr long long kMergeRatio = 4;  // Eq. (1) probe: merge when |B| <= 4 |A remaining|, else binary search
+constexpr int kMergeRatioHash = 1;    // ... and when |B| <= 1 |A remaining| if B has a hash set, else hash probes
 constexpr uint32_t NULL_PAGE = 0xffffffffu;
 constexpr int ERR_STACK = 1;
 
@@ -67,6 +68,33 @@ __device__ __forceinline__ int lower_bound_dev(const int32_t* __restrict__ B, in
   return base;
 }
 
+// w in N(v) by v's adjacency hash set (graph.cu build_hash_index): T_v = T > 0 slots at
+// slots[h0 ..), w at or after its home slot, linear probing, EMPTY = -1.  Reads aligned
+// 16-byte groups of 4 slots; an EMPTY at or after the home slot ends a miss.
+__device__ __forceinline__ unsigned hash_home(unsigned T, int w) {
+  return ((unsigned)w * 2654435769u) >> (__clz(T) + 1);  // >> (32 - log2 T)
+}
+// one group: 1 = hit, 0 = miss, -1 = undecided (group full, no hit)
+__device__ __forceinline__ int hash_group(const int4 q, int w, unsigned skip) {
+  if (q.x == w || q.y == w || q.z == w || q.w == w) return 1;
+  const bool empty = (skip < 1 && q.x < 0) || (skip < 2 && q.y < 0) || (skip < 3 && q.z < 0) || q.w < 0;
+  return empty ? 0 : -1;
+}
+// continue a probe at group g (after an undecided group)
+__device__ __noinline__ bool hash_tail(const int32_t* __restrict__ slots, long long h0, unsigned T, int w, unsigned g) {
+  for (;;) {
+    g = (g + 4) & (T - 1);
+    const int r = hash_group(__ldg(reinterpret_cast<const int4*>(slots + h0 + g)), w, 0);
+    if (r >= 0) return r != 0;
+  }
+}
+__device__ __forceinline__ bool hash_contains(const int32_t* __restrict__ slots, long long h0, unsigned T, int w) {
+  const unsigned s = hash_home(T, w);
+  const int r = hash_group(__ldg(reinterpret_cast<const int4*>(slots + h0 + (s & ~3u))), w, s & 3u);
+  if (r >= 0) return r != 0;
+  return hash_tail(slots, h0, T, w, s & ~3u);
+}
+
 // Same result with power-of-two steps (trip count depends only on n: no divergence).
 __device__ __forceinline__ int lower_bound_pow2(const int32_t* __restrict__ B, int n, int v) {
   if (n <= 0) return 0;
@@ -85,12 +113,12 @@ __device__ __forceinline__ int lower_bound_pow2(const int32_t* __restrict__ B, i
 // atomicCAS / atomicExch handshakes on the -1 sentinel.
 struct Queue {
   QSlot* slots;
-  uint64_t cap;
+  uint64_t nslots;  // ring size, a power of two >= the capacity P.qcap (the `free` counter bounds occupancy)
   unsigned long long *head, *tail, *avail, *free_;
 };
 
 __device__ __forceinline__ Queue make_queue(const KParams& P) {
-  return Queue{P.slots, P.qcap, ctr(P, C_QHEAD), ctr(P, C_QTAIL), ctr(P, C_QAVAIL), ctr(P, C_QFREE)};
+  return Queue{P.slots, P.qslots, ctr(P, C_QHEAD), ctr(P, C_QTAIL), ctr(P, C_QAVAIL), ctr(P, C_QFREE)};
 }
 
 // lane 0: reserve r consecutive tickets; returns ~0 if the queue is full (enqueue -> false).
@@ -105,7 +133,7 @@ __device__ __forceinline__ unsigned long long q_reserve(const Queue& q, int r) {
 
 // one lane: write task into the slot of ticket t and publish it
 __device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, int v1, int v2, int v3) {
-  QSlot* s = q.slots + (t % q.cap);
+  QSlot* s = q.slots + (t & (q.nslots - 1));
   unsigned want = (unsigned)t;
   while (ld_acquire_u32(&s->seq) != want) __nanosleep(32);
   volatile QSlot* vs = s;
@@ -124,14 +152,14 @@ __device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3)
     return false;
   }
   unsigned long long h = atomicAdd(q.head, 1ull);
-  QSlot* s = q.slots + (h % q.cap);
+  QSlot* s = q.slots + (h & (q.nslots - 1));
   unsigned want = (unsigned)(h + 1);
   while (ld_acquire_u32(&s->seq) != want) __nanosleep(32);
   volatile QSlot* vs = s;
   v1 = vs->v1;
   v2 = vs->v2;
   v3 = vs->v3;
-  st_release_u32(&s->seq, (unsigned)(h + q.cap));
+  st_release_u32(&s->seq, (unsigned)(h + q.nslots));
   atomicAdd(q.free_, 1ull);
   return true;
 }

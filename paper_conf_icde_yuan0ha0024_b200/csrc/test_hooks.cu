@@ -128,10 +128,11 @@ int cuda_fail(cudaError_t e, const char* what) {
   return fail(TDFS_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
-__global__ void init_q(QSlot* slots, unsigned long long cap, unsigned long long base, unsigned long long* ctrs) {
-  for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < cap;
+__global__ void init_q(QSlot* slots, unsigned long long cap, unsigned long long nslots, unsigned long long base,
+                       unsigned long long* ctrs) {
+  for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < nslots;
        s += (unsigned long long)gridDim.x * blockDim.x) {
-    slots[s].seq = (unsigned)(base + ((s + cap - (base % cap)) % cap));
+    slots[s].seq = (unsigned)(base + ((s + nslots - (base % nslots)) % nslots));
     slots[s].v1 = slots[s].v2 = slots[s].v3 = -1;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -157,7 +158,9 @@ extern "C" int tdfs_test_queue(int device, int mode, int n_warps, int64_t cap_ta
   unsigned long long* ctrs = nullptr;
   int32_t *din = nullptr, *dout = nullptr;
   size_t nin = (size_t)std::max<int64_t>(n_in, 1);
-  e = cudaMalloc(&slots, sizeof(QSlot) * (size_t)cap_tasks);
+  unsigned long long nslots = 1;
+  while (nslots < (unsigned long long)cap_tasks) nslots <<= 1;
+  e = cudaMalloc(&slots, sizeof(QSlot) * (size_t)nslots);
   if (e == cudaSuccess) e = cudaMalloc(&ctrs, sizeof(unsigned long long) * (C_NUM * kCounterStride + 2));
   if (e == cudaSuccess) e = cudaMalloc(&din, sizeof(int32_t) * 3 * nin);
   if (e == cudaSuccess) e = cudaMalloc(&dout, sizeof(int32_t) * 3 * nin);
@@ -167,11 +170,12 @@ extern "C" int tdfs_test_queue(int device, int mode, int n_warps, int64_t cap_ta
   }
   cudaMemset(ctrs, 0, sizeof(unsigned long long) * (C_NUM * kCounterStride + 2));
   if (n_in) cudaMemcpy(din, h_in, sizeof(int32_t) * 3 * n_in, cudaMemcpyHostToDevice);
-  init_q<<<64, 256>>>(slots, (unsigned long long)cap_tasks, ticket_base, ctrs);
+  init_q<<<64, 256>>>(slots, (unsigned long long)cap_tasks, nslots, ticket_base, ctrs);
   KParams P;
   std::memset(&P, 0, sizeof(P));
   P.slots = slots;
   P.qcap = (uint64_t)cap_tasks;
+  P.qslots = nslots;
   P.ctr = ctrs;
   unsigned long long* d_nout = ctrs + C_NUM * kCounterStride;
   unsigned long long* d_nenq = d_nout + 1;

@@ -175,6 +175,28 @@ def test_hub_bitmaps_do_not_change_results():
         assert U.count(g, q, "auto") == U.count(g, q, "auto", flags=M.TDFS_RUN_NO_HUB_BITMAP | 4 | 8), name
 
 
+def test_hash_index_does_not_change_results(monkeypatch):
+    """Per-vertex adjacency hash sets replace binary searches of
+    non-hub operands; counts equal the oracle with the index on (default threshold and
+    every vertex hashed), off (TDFS_RUN_NO_HASH) and with hubs probed by hash too."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    g = T.rmat(10, 16, 6)
+    assert int(np.bincount(g.edges.reshape(-1)).max()) >= 256  # hubs (bitmaps) and hashed lists both occur
+    names = ["triangle", "c4", "diamond", "tailed_triangle", "k4", "house"]
+    ref = {n: O.count(g, T.query(n), "auto", threads=THREADS) for n in names}
+    for min_deg in ("32", "1"):
+        monkeypatch.setenv("TDFS_HASH_MIN_DEG", min_deg)
+        h = M.tdfs_load_edges(g.n, g.edges)
+        for byref in ("1", "0"):  # leaf set F referenced in place vs materialised in shared memory
+            monkeypatch.setenv("TDFS_BYREF", byref)
+            for n in names:
+                p = M.plan_from_query(T.query(n))
+                for fl in (0, M.TDFS_RUN_NO_HUB_BITMAP, M.TDFS_RUN_NO_HASH, M.TDFS_RUN_NO_HASH | M.TDFS_RUN_NO_LEAF_STAGE,
+                           M.TDFS_RUN_NO_HUB_BITMAP | M.TDFS_RUN_NO_LEAF_STAGE | 4):
+                    assert M.tdfs_count(h, p, M.default_opts(flags=fl)) == ref[n], (n, min_deg, byref, fl)
+        h.free()
+
+
 def test_chunk_queue_grid_invariance():
     rmat12 = graph("r10")
     q = T.query("house")
