@@ -28,8 +28,11 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // list and staged in shared memory; each leaf is then
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
-constexpr int kLeafStage = 512;
-constexpr int64_t kHashMinDeg = 32;  // lists shorter than this are searched (they span <= 2 cache lines)  // default shared-memory ids per warp for the leaf set F
+constexpr int kLeafStage = 512;  // default shared-memory ids per warp for the leaf set F
+// Adjacency hash index: off by default (measured slower than cached binary search on the
+// L2-resident config 2); TDFS_HASH_MIN_DEG=d (e.g. 32) at load time builds it for
+// non-hub vertices of degree >= d.
+constexpr int64_t kHashMinDeg = 0;
 struct DevPlan {
   int32_t k;
   int32_t order[kMaxK];          // query vertex at position p (enumerate output mapping)
@@ -82,9 +85,11 @@ struct Graph {
 };
 
 // ---------------------------------------------------------------- device job
-struct QSlot {                // one task of Q_task, 16 bytes (PAPER.md:191 uses 3 ints)
-  int32_t v1, v2, v3;
+struct QSlot {                // one task of Q_task, 32 bytes (one sector; PAPER.md:191 uses 3 ints)
+  int32_t v1, v2, v3;         // <v1,v2,-2> edge task, <v1,v2,v3> 3-prefix task
+  int32_t v4;                 // -1, or the id range end of a range task <v1,v2,lo,hi>
   uint32_t seq;               // ticket handshake: == t free for ticket t, == t+1 full for ticket t
+  uint32_t pad[3];
 };
 
 enum CounterIdx {            // each counter on its own 128-byte line
@@ -130,6 +135,11 @@ struct KParams {
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
   int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
+  int32_t range_split;
+  int32_t range_min, range_maxt;  // range tasks: >= range_min siblings each, <= range_maxt tasks per split
+  int32_t range_mode;          // 0 auto (slice unless position 2's list is reused), 1 slice, 2 whole list
+  int32_t reuse2_used;         // a later position / the leaf set reuses position 2's list (range tasks build it whole)         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling)
+  int32_t leaf_flat;           // staged leaves: flattened batch streams (else one leaf at a time)
   int32_t lf_byref;            // leaf staging: reference F in place when the plan allows (else materialise)
   int32_t lf_cost_g;
   int32_t lf_cost_h;           // leaf staging cost model: extra cost of a hash probe over a bitmap probe           // leaf staging cost model: one dependent global load in shared-memory steps

@@ -55,6 +55,9 @@ struct Ctx {
   unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
   int* sF;                  // this warp's shared-memory stage for the leaf set F (P.fcap ints)
+  int w2lo, w2hi;           // range task: its level-2 candidates are the ids in [w2lo, w2hi) (warp-uniform)
+  int w2mode;               // 0 no range task; 1 level 2 built as the slice only; 2 built whole, iterated in the slice
+  int end2;                 // mode 2: iteration end index of level 2 (INT_MAX otherwise)
 };
 
 __device__ __forceinline__ int getS(int sreg, int p) { return __shfl_sync(FULL, sreg, p); }
@@ -162,7 +165,9 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       hT = (unsigned)(__ldg(P.hoff + sj + 1) - hb);
     }
   }
-  if (STATS && MODE_OUT != 3) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
+  // a range task re-extends part of a level-2 list its splitter already counted (STATS only)
+  const bool counted = STATS && MODE_OUT != 3 && !(d == 2 && c.w2mode != 0);
+  if (counted) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
     const bool mine = (bm_all >> lane) & 1u;
     unsigned long long wb = 0;
     if (mine) wb = (unsigned long long)(4 * (__ldg(P.offs + c.sreg + 1) - __ldg(P.offs + c.sreg)) + 16);
@@ -171,9 +176,13 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   }
   // constraint window [lo, hi)
   const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
-  const int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
-  const int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
-  if (STATS && MODE_OUT != 3) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
+  int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
+  int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
+  if (d == 2 && c.w2mode == 1) {  // range task: only the level-2 candidates in [w2lo, w2hi)
+    lo = max(lo, c.w2lo);
+    hi = min(hi, c.w2hi);
+  }
+  if (counted) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
     const bool mine = (bm_all >> lane) & 1u;
     unsigned wlen = UINT_MAX;
     if (mine && lo < hi) {
@@ -248,7 +257,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       }
     }
     const long long total = len - __popc(__ballot_sync(FULL, hit));
-    if (STATS && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
+    if (counted && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
     return total;
   }
 
@@ -368,7 +377,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     total += cnt;
   }
   if (MODE_OUT == 3) __syncwarp();
-  if (STATS && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
+  if (counted && d < kVF && lane == d) c.lnodes += (unsigned long long)total;
   return total;
 }
 
@@ -537,6 +546,131 @@ __device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, const FRef& fr
   return total;
 }
 
+// per-lane lower_bound of v in the sorted F[lo, hi) (shared or global memory)
+__device__ __forceinline__ int lane_lower_bound(const int* F, int lo, int hi, int v) {
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (F[mid] < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// w in N(x): hub bitmap row, else hash set, else binary search of adj[b0, b1) (short lists)
+__device__ __forceinline__ bool vertex_has(const KParams& P, int hid, long long hb, unsigned hT, long long b0,
+                                           long long b1, int w) {
+  if (hid >= 0) return (__ldg(P.hub_bits + (long long)hid * P.hub_words + (w >> 5)) >> (w & 31)) & 1u;
+  if (hT) return hash_contains(P.hslots, hb, hT, w);
+  const int n = (int)(b1 - b0);
+  const int pos = lower_bound_dev(P.adj + b0, n, w);
+  return pos < n && __ldg(P.adj + b0 + pos) == w;
+}
+
+// largest lane j with pre[j] <= idx (pre non-decreasing over lanes, INT_MAX past the batch)
+__device__ __forceinline__ int seg_of(int pre, int idx) {
+  int j = 0;
+#pragma unroll
+  for (int s = 16; s > 0; s >>= 1)
+    if (__shfl_sync(FULL, pre, j + s) <= idx) j += s;
+  return j;
+}
+
+__device__ __forceinline__ int warp_excl_scan(int v, int lane) {
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  return x - v;
+}
+
+// A whole batch of nb <= 32 staged leaves at once: lane j
+// holds leaf x_j = S[k-2] and N(x_j)'s metadata.  The count is only summed, so the batch's
+// work is flattened into two load-balanced streams of (leaf, element) pairs:
+//   A: leaves where streaming F is cheaper: elements F[lo_j .. hi_j), each probed in N(x_j)
+//      (bitmap / hash set / binary search of a short list);
+//   B: the others: elements of N(x_j), each tested against [F_min_j, F_max_j] and probed in
+//      F (y's bitmap / hash set when F is referenced, else a shared-memory binary search).
+// Every lane takes one pair per round whatever the leaves' sizes -- no per-leaf rounds.
+template <bool STATS>
+__device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr, int nF, int nb, int x,
+                                const VMeta& m) {
+  const DevPlan& pl = P.plan;
+  const int lane = c.lane;
+  const int* F = fr.F;
+  const bool byref = fr.hid >= 0 || fr.hT;
+  const bool act = lane < nb;
+  int lo = 0, hi = nF;
+  if (act && pl.lf_lo_var) lo = lane_lower_bound(F, 0, nF, x + 1);
+  if (act && pl.lf_hi_var) hi = lane_lower_bound(F, lo, nF, x);
+  if (!pl.lf_var) {
+    long long cnt = (act && lo < hi) ? hi - lo : 0;
+    if (cnt && pl.lf_inj_var) {
+      const int i = lane_lower_bound(F, lo, hi, x);
+      cnt -= (i < hi && F[i] == x) ? 1 : 0;
+    }
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
+    return cnt;
+  }
+  const int a = (act && lo < hi) ? hi - lo : 0;
+  const int b = act ? (int)(m.b1 - m.b0) : 0;
+  int wA = 0, wB = 0;
+  if (a > 0 && b > 0) {
+    const int lgb = 32 - __clz(b), lga = 32 - __clz(a);
+    const long long uA = m.hid >= 0 ? 4 : m.hT ? 4 + P.lf_cost_h : 3 + lgb;
+    const long long uB = byref ? (fr.hid >= 0 ? 4 : 4 + P.lf_cost_h) : 3 + (lga >> 1);
+    if ((long long)a * uA <= (long long)b * uB) wA = a;
+    else wB = b;
+  }
+  const int fmin = wB ? F[lo] : 0, fmax = wB ? F[hi - 1] : 0;
+  long long total = 0;
+  // stream A: (j, F[lo_j + i]) probed in N(x_j)
+  {
+    const int pre = warp_excl_scan(wA, lane);
+    const int tot = __shfl_sync(FULL, pre + wA, 31);
+    const int preS = act ? pre : INT_MAX;
+    for (int base = 0; base < tot; base += 32) {
+      const int idx = base + lane;
+      const int j = seg_of(preS, idx);
+      const int i = idx - __shfl_sync(FULL, pre, j);
+      const int lj = __shfl_sync(FULL, lo, j);
+      const int hidj = __shfl_sync(FULL, m.hid, j);
+      const unsigned hTj = __shfl_sync(FULL, m.hT, j);
+      const long long hbj = __shfl_sync(FULL, m.hb, j);
+      const long long b0j = __shfl_sync(FULL, m.b0, j), b1j = __shfl_sync(FULL, m.b1, j);
+      bool ok = false;
+      if (idx < tot) ok = vertex_has(P, hidj, hbj, hTj, b0j, b1j, F[lj + i]);
+      total += __popc(__ballot_sync(FULL, ok));
+    }
+  }
+  // stream B: (j, N(x_j)[i]) tested against F
+  {
+    const int pre = warp_excl_scan(wB, lane);
+    const int tot = __shfl_sync(FULL, pre + wB, 31);
+    const int preS = act ? pre : INT_MAX;
+    for (int base = 0; base < tot; base += 32) {
+      const int idx = base + lane;
+      const int j = seg_of(preS, idx);
+      const int i = idx - __shfl_sync(FULL, pre, j);
+      const long long b0j = __shfl_sync(FULL, m.b0, j);
+      const int fminj = __shfl_sync(FULL, fmin, j), fmaxj = __shfl_sync(FULL, fmax, j);
+      const int loj = __shfl_sync(FULL, lo, j), hij = __shfl_sync(FULL, hi, j);
+      bool ok = false;
+      if (idx < tot) {
+        const int v = __ldg(P.adj + b0j + i);
+        if (v >= fminj && v <= fmaxj) {
+          if (fr.hid >= 0) ok = (__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
+          else if (fr.hT) ok = hash_contains(P.hslots, fr.hb, fr.hT, v);
+          else ok = F[smem_lower_bound(F, loj, hij, v)] == v;  // index < hij since v <= F[hij - 1]
+        }
+      }
+      total += __popc(__ballot_sync(FULL, ok));
+    }
+  }
+  return total;
+}
+
 // Stage F for the level-(k-2) list just built (see FRef).  Returns |F|, or -2 when F
 // would have to be materialised and exceeds the shared-memory stage (generic per leaf).
 template <bool STATS>
@@ -588,13 +722,41 @@ __device__ long long split_level2(const KParams& P, Ctx<STATS>& c, const Queue& 
   return size;
 }
 
+// Timeout split of level 2 when its children are leaves (k = 4): instead of one task per
+// remaining sibling (each a single Eq. (1) intersection), push at most 32 range tasks
+// <S0, S1, lo, hi>, each covering >= 32 consecutive siblings C[i .. i+g) by id range
+// [C[i], C[i+g]) (the last one up to this list's own bound w2hi).  A receiver rebuilds
+// its slice of level 2 with that extra window, stages the leaf set once and processes
+// the leaves in flat batches.  Returns false if the queue is full.
+template <bool STATS>
+__device__ bool split_level2_ranges(const KParams& P, Ctx<STATS>& c, const Queue& q, int from, int size) {
+  const int lane = c.lane;
+  const uint32_t* table = c.tables;  // level index 0 = position 2
+  const int rem = size - from;
+  const int g = max(P.range_min, (rem + P.range_maxt - 1) / P.range_maxt);
+  const int ntask = (rem + g - 1) / g;
+  const int i0 = from + lane * g, i1 = i0 + g;
+  int lo = 0, hi = c.w2hi;
+  if (lane < ntask) lo = paged_read(P, table, i0);
+  if (lane < ntask && i1 < size) hi = paged_read(P, table, i1);
+  const unsigned mask = ntask >= 32 ? FULL : ((1u << ntask) - 1u);
+  const int s0 = getS(c.sreg, 0), s1 = getS(c.sreg, 1);
+  if (!q_push_warp(P, q, mask, s0, s1, lo, lane, hi)) {
+    if (STATS && lane == 0) c.qfull++;
+    return false;
+  }
+  if (STATS && lane == 0) c.enq += ntask;
+  return true;
+}
+
 // Depth-first search below a prefix S[0..start-1] (Alg. 4 l.7-28).
 // Returns false on error.
 template <int MODE, bool STATS>
 __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) {
   const int k = P.plan.k;
   const int lane = c.lane;
-  const bool own2 = (start == 2);  // level 2 built by this warp (not a <v1,v2,v3> task)
+  // level 2 built whole by this warp (not a <v1,v2,v3> task, not a range task's slice): reusable
+  const bool own2 = (start == 2) && c.w2mode != 1;
   if (start == k - 1) {
     long long n = (MODE == 1) ? extend<2, STATS>(P, c, start, own2) : extend<1, STATS>(P, c, start, own2);
     c.count += (unsigned long long)n;
@@ -608,6 +770,12 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
   long long sz = extend<0, STATS>(P, c, d, own2);
   if (sz < 0) return false;
   if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
+  if (start == 2 && c.w2mode == 2) {  // range task over a whole level-2 list: iterate [w2lo, w2hi) only
+    const long long ib = warp_paged_lower_bound(P, c.tables, 0, sz, c.w2lo, lane);
+    const long long ie = c.w2hi < INT_MAX ? warp_paged_lower_bound(P, c.tables, ib, sz, c.w2hi, lane) : sz;
+    if (lane == d) c.liter = (int)ib;
+    c.end2 = (int)ie;
+  }
   if (use_lf && d == k - 2) {
     nF = sz >= 2 ? stage_leaf_set(P, c, own2, fr) : -1;
     if (nF == 0 && lane == d) c.liter = (int)sz;  // F empty: no leaf below this list
@@ -615,11 +783,26 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
   bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
   for (;;) {
     const int it = __shfl_sync(FULL, c.liter, d);
-    const int size = __shfl_sync(FULL, c.lsize, d);
+    const int size = d == 2 ? min(__shfl_sync(FULL, c.lsize, d), c.end2) : __shfl_sync(FULL, c.lsize, d);
     if (it < size) {
       if (d == 2 && !grace && timed_out(P, c)) {
         // timeout: push the current and all remaining siblings, then backtrack
         if (STATS && lane == 0) c.touts++;
+        if (k == 4 && P.range_split) {
+          // <= 32 remaining siblings finish in place (tasks strictly shrink: progress at tau = 0)
+          if (size - it <= P.range_min) {
+            if (lane == 0) c.t0 = globaltimer();
+            grace = true;
+            continue;
+          }
+          if (split_level2_ranges(P, c, q, it, size)) {
+            if (lane == d) c.liter = size;
+            continue;
+          }
+          if (lane == 0) c.t0 = globaltimer();  // queue full: continue in place
+          grace = true;
+          continue;
+        }
         long long upto = split_level2(P, c, q, it, size);
         if (upto >= size) {
           if (lane == d) c.liter = size;
@@ -638,10 +821,12 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         // loaded by one lane each (independent loads), then each leaf is one |F ∩ N(x)|
         const int nb = min(32, size - it);
         const int vl = lane < nb ? paged_read(P, table, it + lane) : 0;
-        VMeta ml;
+        VMeta ml = {0, 0, 0, 0u, -1};
         if (lane < nb) ml = load_vmeta(P, vl);
         long long n = 0;
-        for (int j = 0; j < nb; j++) n += leaf_staged(P, c, fr, nF, __shfl_sync(FULL, vl, j), shfl_vmeta(ml, j));
+        if (P.leaf_flat) n = leaf_batch(P, c, fr, nF, nb, vl, ml);
+        else
+          for (int j = 0; j < nb; j++) n += leaf_staged(P, c, fr, nF, __shfl_sync(FULL, vl, j), shfl_vmeta(ml, j));
         c.count += (unsigned long long)n;
         if (lane == d) c.liter = it + nb;
         continue;
@@ -758,6 +943,10 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.t0 = 0;
   c.lnodes = 0;
   c.wbytes = c.sbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
+  c.w2lo = 0;
+  c.w2hi = INT_MAX;
+  c.w2mode = 0;
+  c.end2 = INT_MAX;
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
   extern __shared__ int smem_stage[];
   c.sF = smem_stage + (threadIdx.x >> 5) * P.fcap;
@@ -790,9 +979,9 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
       busy = true;
     }
     // 1. Q_task first
-    int got = 0, t1 = 0, t2 = 0, t3 = 0;
+    int got = 0, t1 = 0, t2 = 0, t3 = 0, t4 = -1;
     if (lane == 0) {
-      got = q_pop(q, t1, t2, t3);
+      got = q_pop(q, t1, t2, t3, t4);
       if (got) c.t0 = globaltimer();
     }
     got = __shfl_sync(FULL, got, 0);
@@ -800,11 +989,23 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
       t1 = __shfl_sync(FULL, t1, 0);
       t2 = __shfl_sync(FULL, t2, 0);
       t3 = __shfl_sync(FULL, t3, 0);
+      t4 = __shfl_sync(FULL, t4, 0);
       if (STATS && lane == 0) c.deq++;
       if (lane == 0) c.sreg = t1;
       if (lane == 1) c.sreg = t2;
       if (lane == 2) c.sreg = t3;
-      if (!dfs<MODE, STATS>(P, c, q, t3 == -2 ? 2 : 3)) {
+      const bool range = t3 >= 0 && t4 >= 0;  // <v1, v2, lo, hi>: level-2 candidates in [lo, hi)
+      if (range) {
+        c.w2lo = t3;
+        c.w2hi = t4;
+        c.w2mode = P.range_mode ? P.range_mode : (P.reuse2_used ? 2 : 1);
+      }
+      const bool ok = dfs<MODE, STATS>(P, c, q, (t3 == -2 || range) ? 2 : 3);
+      c.w2lo = 0;
+      c.w2hi = INT_MAX;
+      c.w2mode = 0;
+      c.end2 = INT_MAX;
+      if (!ok) {
         raise_error(P, ERR_STACK);
         break;
       }
@@ -860,7 +1061,7 @@ __global__ void init_queue_kernel(QSlot* slots, unsigned long long cap, unsigned
        s += (unsigned long long)gridDim.x * blockDim.x) {
     unsigned long long first = base + ((s + cap - (base % cap)) % cap);  // first ticket >= base hitting slot s
     slots[s].seq = (unsigned)first;
-    slots[s].v1 = slots[s].v2 = slots[s].v3 = -1;
+    slots[s].v1 = slots[s].v2 = slots[s].v3 = slots[s].v4 = -1;
   }
 }
 
@@ -1004,6 +1205,9 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   }
   if (o->flags & TDFS_RUN_NO_SHORTCUT)
     for (int i = 0; i < kMaxK; i++) P.plan.shortcut[i] = 0;
+  P.reuse2_used = 0;  // does any later position (or the leaf set) start from position 2's list?
+  for (int i = 3; i <= kVF; i++)
+    if ((i < P.plan.k || i == kVF) && P.plan.reuse[i] == 2) P.reuse2_used = 1;
   P.shard_rank = o->shard_rank;
   P.shard_world = o->shard_world;
   P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
@@ -1024,6 +1228,15 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.lf_cost_g = 6;
   P.lf_cost_h = 2;
   if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
+  P.range_split = 1;
+  P.range_min = 32;
+  P.range_maxt = 32;
+  if (const char* e = getenv("TDFS_RANGE_MIN")) P.range_min = std::max(1, atoi(e));  // tuning knobs (experiments)
+  if (const char* e = getenv("TDFS_RANGE_MAXT")) P.range_maxt = std::min(32, std::max(2, atoi(e)));
+  if (const char* e = getenv("TDFS_RANGE_MODE")) P.range_mode = atoi(e);
+  if (const char* e = getenv("TDFS_RANGE_SPLIT")) P.range_split = atoi(e);  // tuning knob (experiments)
+  P.leaf_flat = 1;
+  if (const char* e = getenv("TDFS_LEAF_FLAT")) P.leaf_flat = atoi(e);  // tuning knob (experiments)
   P.lf_byref = 1;
   if (const char* e = getenv("TDFS_BYREF")) P.lf_byref = atoi(e);  // tuning knob (experiments)
   P.coop_window = 1;

@@ -132,7 +132,7 @@ __device__ __forceinline__ unsigned long long q_reserve(const Queue& q, int r) {
 }
 
 // one lane: write task into the slot of ticket t and publish it
-__device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, int v1, int v2, int v3) {
+__device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, int v1, int v2, int v3, int v4) {
   QSlot* s = q.slots + (t & (q.nslots - 1));
   unsigned want = (unsigned)t;
   while (ld_acquire_u32(&s->seq) != want) __nanosleep(32);
@@ -140,11 +140,12 @@ __device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, 
   vs->v1 = v1;
   vs->v2 = v2;
   vs->v3 = v3;
+  vs->v4 = v4;
   st_release_u32(&s->seq, (unsigned)(t + 1));
 }
 
 // lane 0: Alg. 3 dequeue.  Returns false when empty.
-__device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3) {
+__device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3, int& v4) {
   if (ld_relaxed_s64(q.avail) <= 0) return false;
   long long old = (long long)atomicAdd(q.avail, (unsigned long long)(-1ll));
   if (old <= 0) {
@@ -159,15 +160,16 @@ __device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3)
   v1 = vs->v1;
   v2 = vs->v2;
   v3 = vs->v3;
+  v4 = vs->v4;
   st_release_u32(&s->seq, (unsigned)(h + q.nslots));
   atomicAdd(q.free_, 1ull);
   return true;
 }
 
 // Warp-cooperative push of the tasks held by the lanes in `mask` (lane i pushes
-// <a_i, b_i, c_i>).  Returns false if the queue is full (nothing pushed).
+// <a_i, b_i, c_i, d_i>).  Returns false if the queue is full (nothing pushed).
 __device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, unsigned mask, int a, int b, int c,
-                                           int lane) {
+                                           int lane, int d = -1) {
   int r = __popc(mask);
   if (r == 0) return true;
   unsigned long long t = 0;
@@ -176,7 +178,7 @@ __device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, un
   if (t == ~0ull) return false;
   if (mask >> lane & 1u) {
     unsigned long long my = t + __popc(mask & lanemask_lt());
-    q_publish(q, my, a, b, c);
+    q_publish(q, my, a, b, c, d);
   }
   __syncwarp();
   if (P.trace) {

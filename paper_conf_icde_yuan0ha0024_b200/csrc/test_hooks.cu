@@ -23,8 +23,8 @@ __global__ void queue_test_kernel(KParams P, int mode, const int32_t* in, long l
   const int nw = (gridDim.x * blockDim.x) >> 5;
   const Queue q = make_queue(P);
   auto pop_one = [&]() -> bool {
-    int got = 0, a = 0, b = 0, c = 0;
-    if (lane == 0) got = q_pop(q, a, b, c);
+    int got = 0, a = 0, b = 0, c = 0, d = 0;
+    if (lane == 0) got = q_pop(q, a, b, c, d);
     got = __shfl_sync(FULL, got, 0);
     if (got && lane == 0) {
       unsigned long long i = atomicAdd(n_out, 1ull);
@@ -133,7 +133,7 @@ __global__ void init_q(QSlot* slots, unsigned long long cap, unsigned long long 
   for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < nslots;
        s += (unsigned long long)gridDim.x * blockDim.x) {
     slots[s].seq = (unsigned)(base + ((s + nslots - (base % nslots)) % nslots));
-    slots[s].v1 = slots[s].v2 = slots[s].v3 = -1;
+    slots[s].v1 = slots[s].v2 = slots[s].v3 = slots[s].v4 = -1;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     ctrs[C_QHEAD * kCounterStride] = base;

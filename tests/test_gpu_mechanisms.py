@@ -115,3 +115,25 @@ def test_split_counts_are_tau_invariant_on_skewed_graph():
         assert cnt == ref
         if tau == 0.0:
             assert st["tasks_enqueued"] > 0 and st["tasks_enqueued"] == st["tasks_dequeued"]
+
+
+@pytest.mark.parametrize("range_split", ["1", "0"])
+def test_level2_range_tasks_k4(monkeypatch, range_split):
+    """k = 4: a timed-out level-2 list is split into <= 32 id-range tasks <S0, S1, lo, hi>
+     instead of one task per sibling.  With tau = 0 every level-2
+    step splits; counts, per-level node counts and W (STATS variant) still equal the
+    oracle's, and every pushed task is dequeued exactly once."""
+    monkeypatch.setenv("TDFS_RANGE_SPLIT", range_split)
+    g = T.rmat(11, 12, 4)
+    for name in ("c4", "diamond", "k4", "tailed_triangle"):
+        q = T.query(name)
+        order = O.oracle_order(q)
+        r = O.match(g, q, "auto", order=order, deg_filter=True, threads=8)
+        for kw in (dict(tau_ms=0.0), dict(tau_ms=0.0, blocks=2, warps_per_block=2), dict(tau_ms=0.01)):
+            cnt, st = U.count(g, q, "auto", order=order, stats=True, **kw)
+            assert cnt == r["count"], (name, kw)
+            assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k], (name, kw)
+            assert st["adj_bytes"] == r["W"] and st["stream_bytes"] == r["W_stream"], (name, kw)
+            assert st["tasks_enqueued"] == st["tasks_dequeued"], (name, kw)
+            assert U.count(g, q, "auto", order=order, **kw) == r["count"], (name, kw)
+        assert st["tasks_enqueued"] > 0
