@@ -389,6 +389,56 @@ def tdfs_enumerate(g: GraphHandle, p: PlanHandle, cap: int, opts: Optional[tdfs_
     return res + (s.as_dict(),) if stats else res
 
 
+def tdfs_enumerate_chunks(g: GraphHandle, p: PlanHandle, chunk_cap: int, opts: Optional[tdfs_run_opts] = None,
+                          workspace=None, stream=None):
+    """Enumerate every match in chunks of at most `chunk_cap` tuples, streamed to pinned host
+    memory ("output S").
+
+    Marshalling only -- all matching runs in tdfs_count / tdfs_enumerate.  The initial edge
+    tasks of this caller's shard (opts.shard_rank / shard_world; a multi-GPU rank streams its
+    rank-local output) are refined into round-robin sub-shards (r + W*s of W*S),
+    S sized from one count pass so that each sub-shard's tuples fit one device buffer of
+    chunk_cap * k ints; a sub-shard that still overflows is split in two.  Yields
+    (tuples (n, k) int32 numpy array, total_so_far); tuples are indexed by query vertex id."""
+    torch = _torch()
+    opts = opts or default_opts()
+    if chunk_cap < 1:
+        raise TdfsError(TDFS_E_INVALID_ARG, "chunk_cap must be >= 1")
+    k = p.k
+    base_r, base_w = int(opts.shard_rank), int(opts.shard_world)
+    total = tdfs_count(g, p, opts, workspace=workspace, stream=stream)
+    if total == 0:
+        return
+    out = torch.empty(chunk_cap * k, dtype=torch.int32, device=f"cuda:{g.device}")
+    host = torch.empty(chunk_cap * k, dtype=torch.int32, pin_memory=True)
+    S = max(1, -(-2 * total // chunk_cap))  # ~2x headroom for uneven sub-shards
+    todo = [(base_r + base_w * s, base_w * S) for s in range(S - 1, -1, -1)]
+    done = 0
+    while todo:
+        r, w = todo.pop()
+        if w >= 2**31 - 1:
+            raise TdfsError(TDFS_E_INVALID_ARG, "a single initial edge has more than chunk_cap matches")
+        o = tdfs_run_opts.from_buffer_copy(opts)
+        o.shard_rank, o.shard_world = r, w
+        tot = ctypes.c_uint64(0)
+        nbytes = tdfs_workspace_bytes(g, p, o)
+        ws = _ws_for(g, nbytes, workspace)
+        rc = _lib.tdfs_enumerate(g.ptr, p.ptr, ctypes.byref(o), ws.data_ptr(), ws.numel(), _stream_ptr(stream, g.device),
+                                 out.data_ptr(), int(chunk_cap), ctypes.byref(tot), None)
+        _check(rc, allow=(TDFS_E_OUTPUT_OVERFLOW,))
+        if rc == TDFS_E_OUTPUT_OVERFLOW:  # split this sub-shard in two: r and r + w of 2w
+            todo += [(r + w, 2 * w), (r, 2 * w)]
+            continue
+        n = int(tot.value)
+        if n == 0:
+            continue
+        host[: n * k].copy_(out[: n * k])
+        done += n
+        yield host[: n * k].view(n, k).numpy().copy(), done
+    if done != total:
+        raise TdfsError(TDFS_E_CUDA, f"chunked enumeration produced {done} tuples, count pass {total}")
+
+
 def tdfs_workspace_status(workspace, stream=None, device: int = 0) -> int:
     return _check(_lib.tdfs_workspace_status(workspace.data_ptr(), _stream_ptr(stream, device)))
 

@@ -135,10 +135,12 @@ struct KParams {
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
   int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
+  int32_t smem_fcap;           // shared-memory layout: F ids per warp (the launch's, even when staging is off)
   int32_t range_split;
   int32_t range_min, range_maxt;  // range tasks: >= range_min siblings each, <= range_maxt tasks per split
   int32_t range_mode;          // 0 auto (slice unless position 2's list is reused), 1 slice, 2 whole list
-  int32_t reuse2_used;         // a later position / the leaf set reuses position 2's list (range tasks build it whole)         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling)
+  int32_t reuse2_used;
+  int32_t range_ok;            // the plan uses range tasks (see launch_job)         // a later position / the leaf set reuses position 2's list (range tasks build it whole)         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling)
   int32_t leaf_flat;           // staged leaves: flattened batch streams (else one leaf at a time)
   int32_t lf_byref;            // leaf staging: reference F in place when the plan allows (else materialise)
   int32_t lf_cost_g;

@@ -43,6 +43,22 @@ namespace {
 
 #include "prims.cuh"
 
+// per-leaf entry of a flat leaf batch (shared memory, one per lane of the batch)
+struct LeafMeta {
+  long long b0;  // N(x) = adj[b0, b0 + deg)
+  int deg;
+  int hid;       // hub bitmap row of x, -1 = none
+  int lo, hi;    // F window of this leaf: F[lo, hi)
+};
+// 32 entries + 33 prefix ints, padded to 16 B; with the 2 KB F stage, 16 blocks x 4 warps fit an SM
+constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144;
+__host__ __device__ inline size_t smem_meta_offset(int wpb, int fcap) {
+  return ((size_t)wpb * fcap * sizeof(int) + 15) & ~(size_t)15;
+}
+__host__ __device__ inline size_t smem_bytes(int wpb, int fcap) {
+  return smem_meta_offset(wpb, fcap) + (size_t)wpb * kMetaBytesPerWarp;
+}
+
 // ------------------------------------------------------------ warp context
 template <bool STATS>
 struct Ctx {
@@ -55,6 +71,8 @@ struct Ctx {
   unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
   int* sF;                  // this warp's shared-memory stage for the leaf set F (P.fcap ints)
+  LeafMeta* sMeta;          // this warp's leaf-batch metadata (32 entries) ...
+  int* sPre;                // ... and the batch's exclusive prefix sums (33 ints)
   int w2lo, w2hi;           // range task: its level-2 candidates are the ids in [w2lo, w2hi) (warp-uniform)
   int w2mode;               // 0 no range task; 1 level 2 built as the slice only; 2 built whole, iterated in the slice
   int end2;                 // mode 2: iteration end index of level 2 (INT_MAX otherwise)
@@ -556,25 +574,6 @@ __device__ __forceinline__ int lane_lower_bound(const int* F, int lo, int hi, in
   return lo;
 }
 
-// w in N(x): hub bitmap row, else hash set, else binary search of adj[b0, b1) (short lists)
-__device__ __forceinline__ bool vertex_has(const KParams& P, int hid, long long hb, unsigned hT, long long b0,
-                                           long long b1, int w) {
-  if (hid >= 0) return (__ldg(P.hub_bits + (long long)hid * P.hub_words + (w >> 5)) >> (w & 31)) & 1u;
-  if (hT) return hash_contains(P.hslots, hb, hT, w);
-  const int n = (int)(b1 - b0);
-  const int pos = lower_bound_dev(P.adj + b0, n, w);
-  return pos < n && __ldg(P.adj + b0 + pos) == w;
-}
-
-// largest lane j with pre[j] <= idx (pre non-decreasing over lanes, INT_MAX past the batch)
-__device__ __forceinline__ int seg_of(int pre, int idx) {
-  int j = 0;
-#pragma unroll
-  for (int s = 16; s > 0; s >>= 1)
-    if (__shfl_sync(FULL, pre, j + s) <= idx) j += s;
-  return j;
-}
-
 __device__ __forceinline__ int warp_excl_scan(int v, int lane) {
   int x = v;
 #pragma unroll
@@ -589,7 +588,7 @@ __device__ __forceinline__ int warp_excl_scan(int v, int lane) {
 // holds leaf x_j = S[k-2] and N(x_j)'s metadata.  The count is only summed, so the batch's
 // work is flattened into two load-balanced streams of (leaf, element) pairs:
 //   A: leaves where streaming F is cheaper: elements F[lo_j .. hi_j), each probed in N(x_j)
-//      (bitmap / hash set / binary search of a short list);
+//      (hub bitmap, else binary search);
 //   B: the others: elements of N(x_j), each tested against [F_min_j, F_max_j] and probed in
 //      F (y's bitmap / hash set when F is referenced, else a shared-memory binary search).
 // Every lane takes one pair per round whatever the leaves' sizes -- no per-leaf rounds.
@@ -618,47 +617,79 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   int wA = 0, wB = 0;
   if (a > 0 && b > 0) {
     const int lgb = 32 - __clz(b), lga = 32 - __clz(a);
-    const long long uA = m.hid >= 0 ? 4 : m.hT ? 4 + P.lf_cost_h : 3 + lgb;
+    const long long uA = m.hid >= 0 ? 4 : 3 + lgb;
     const long long uB = byref ? (fr.hid >= 0 ? 4 : 4 + P.lf_cost_h) : 3 + (lga >> 1);
     if ((long long)a * uA <= (long long)b * uB) wA = a;
     else wB = b;
   }
-  const int fmin = wB ? F[lo] : 0, fmax = wB ? F[hi - 1] : 0;
+  // the batch's per-leaf entries go to shared memory: a lane then reads its current leaf's
+  // entry only when it moves to the next leaf (no warp-wide shuffles per element)
+  LeafMeta* meta = c.sMeta;
+  int* pre = c.sPre;
+  if (act) {
+    LeafMeta e;
+    e.b0 = m.b0;
+    e.deg = b;
+    e.hid = m.hid;
+    e.lo = lo;
+    e.hi = hi;
+    meta[lane] = e;
+  }
   long long total = 0;
   // stream A: (j, F[lo_j + i]) probed in N(x_j)
   {
-    const int pre = warp_excl_scan(wA, lane);
-    const int tot = __shfl_sync(FULL, pre + wA, 31);
-    const int preS = act ? pre : INT_MAX;
+    const int p = warp_excl_scan(wA, lane);
+    const int tot = __shfl_sync(FULL, p + wA, 31);
+    __syncwarp();
+    pre[lane] = act ? p : tot;
+    if (lane == 0) pre[32] = tot;
+    __syncwarp();
+    int j = -1, jn = 0, pj = 0, lj = 0, hidj = -1, degj = 0;
+    long long b0j = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
-      const int j = seg_of(preS, idx);
-      const int i = idx - __shfl_sync(FULL, pre, j);
-      const int lj = __shfl_sync(FULL, lo, j);
-      const int hidj = __shfl_sync(FULL, m.hid, j);
-      const unsigned hTj = __shfl_sync(FULL, m.hT, j);
-      const long long hbj = __shfl_sync(FULL, m.hb, j);
-      const long long b0j = __shfl_sync(FULL, m.b0, j), b1j = __shfl_sync(FULL, m.b1, j);
       bool ok = false;
-      if (idx < tot) ok = vertex_has(P, hidj, hbj, hTj, b0j, b1j, F[lj + i]);
+      if (idx < tot) {
+        if (idx >= jn) {  // move to the leaf holding idx (per lane, shared-memory reads)
+          do { ++j; jn = pre[j + 1]; } while (jn <= idx);
+          pj = pre[j];
+          const LeafMeta e = meta[j];
+          lj = e.lo; hidj = e.hid; degj = e.deg; b0j = e.b0;
+        }
+        const int w = F[lj + idx - pj];
+        if (hidj >= 0) {
+          ok = (__ldg(P.hub_bits + (long long)hidj * P.hub_words + (w >> 5)) >> (w & 31)) & 1u;
+        } else {
+          const int pos = lower_bound_dev(P.adj + b0j, degj, w);
+          ok = pos < degj && __ldg(P.adj + b0j + pos) == w;
+        }
+      }
       total += __popc(__ballot_sync(FULL, ok));
     }
   }
   // stream B: (j, N(x_j)[i]) tested against F
   {
-    const int pre = warp_excl_scan(wB, lane);
-    const int tot = __shfl_sync(FULL, pre + wB, 31);
-    const int preS = act ? pre : INT_MAX;
+    const int p = warp_excl_scan(wB, lane);
+    const int tot = __shfl_sync(FULL, p + wB, 31);
+    __syncwarp();
+    pre[lane] = act ? p : tot;
+    if (lane == 0) pre[32] = tot;
+    __syncwarp();
+    int j = -1, jn = 0, pj = 0, loj = 0, hij = 0, fminj = 0, fmaxj = 0;
+    long long b0j = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
-      const int j = seg_of(preS, idx);
-      const int i = idx - __shfl_sync(FULL, pre, j);
-      const long long b0j = __shfl_sync(FULL, m.b0, j);
-      const int fminj = __shfl_sync(FULL, fmin, j), fmaxj = __shfl_sync(FULL, fmax, j);
-      const int loj = __shfl_sync(FULL, lo, j), hij = __shfl_sync(FULL, hi, j);
       bool ok = false;
       if (idx < tot) {
-        const int v = __ldg(P.adj + b0j + i);
+        if (idx >= jn) {
+          do { ++j; jn = pre[j + 1]; } while (jn <= idx);
+          pj = pre[j];
+          const LeafMeta e = meta[j];
+          loj = e.lo; hij = e.hi; b0j = e.b0;
+          fminj = F[loj];
+          fmaxj = F[hij - 1];
+        }
+        const int v = __ldg(P.adj + b0j + idx - pj);
         if (v >= fminj && v <= fmaxj) {
           if (fr.hid >= 0) ok = (__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
           else if (fr.hT) ok = hash_contains(P.hslots, fr.hb, fr.hT, v);
@@ -668,6 +699,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
       total += __popc(__ballot_sync(FULL, ok));
     }
   }
+  __syncwarp();
   return total;
 }
 
@@ -788,7 +820,7 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
       if (d == 2 && !grace && timed_out(P, c)) {
         // timeout: push the current and all remaining siblings, then backtrack
         if (STATS && lane == 0) c.touts++;
-        if (k == 4 && P.range_split) {
+        if (k == 4 && P.range_split && P.range_ok) {
           // <= 32 remaining siblings finish in place (tasks strictly shrink: progress at tau = 0)
           if (size - it <= P.range_min) {
             if (lane == 0) c.t0 = globaltimer();
@@ -929,7 +961,7 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
 // The persistent matching kernel.  MODE 0 = count, 1 = enumerate.
 template <int MODE, bool STATS>
 #ifndef TDFS_MIN_BLOCKS
-#define TDFS_MIN_BLOCKS 16
+#define TDFS_MIN_BLOCKS 12  // 40 registers: measured best of 8..16 on config 2
 #endif
 __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParams P) {
   const int lane = threadIdx.x & 31;
@@ -950,6 +982,12 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
   extern __shared__ int smem_stage[];
   c.sF = smem_stage + (threadIdx.x >> 5) * P.fcap;
+  {
+    char* meta = reinterpret_cast<char*>(smem_stage) + smem_meta_offset(blockDim.x >> 5, P.smem_fcap) +
+                 (threadIdx.x >> 5) * kMetaBytesPerWarp;
+    c.sMeta = reinterpret_cast<LeafMeta*>(meta);
+    c.sPre = reinterpret_cast<int*>(meta + 32 * sizeof(LeafMeta));
+  }
   const Queue q = make_queue(P);
   int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
   unsigned long long* cursor = ctr(P, C_CURSOR);
@@ -1100,7 +1138,7 @@ int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int
   (void)device;
   int nb = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, pick_kernel(enumerate ? 1 : 0, stats), wpb * 32,
-                                                                (size_t)wpb * fcap * sizeof(int));
+                                                                smem_bytes(wpb, fcap));
   if (e != cudaSuccess) return cuda_fail(e, "occupancy");
   *out = std::max(1, nb);
   return TDFS_OK;
@@ -1208,6 +1246,9 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.reuse2_used = 0;  // does any later position (or the leaf set) start from position 2's list?
   for (int i = 3; i <= kVF; i++)
     if ((i < P.plan.k || i == kVF) && P.plan.reuse[i] == 2) P.reuse2_used = 1;
+  // range tasks rebuild level 2 per task: worth it unless the leaves are intersections that
+  // start from the splitter's level-2 list (k4: per-sibling tasks measured 86 vs 100 ms)
+  P.range_ok = !(P.reuse2_used && P.plan.lf_var);
   P.shard_rank = o->shard_rank;
   P.shard_world = o->shard_world;
   P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
@@ -1225,6 +1266,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.E = L.E;
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
+  P.smem_fcap = L.fcap;
   P.lf_cost_g = 6;
   P.lf_cost_h = 2;
   if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
@@ -1234,6 +1276,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   if (const char* e = getenv("TDFS_RANGE_MIN")) P.range_min = std::max(1, atoi(e));  // tuning knobs (experiments)
   if (const char* e = getenv("TDFS_RANGE_MAXT")) P.range_maxt = std::min(32, std::max(2, atoi(e)));
   if (const char* e = getenv("TDFS_RANGE_MODE")) P.range_mode = atoi(e);
+  if (const char* e = getenv("TDFS_RANGE_FORCE")) P.range_ok = atoi(e);
   if (const char* e = getenv("TDFS_RANGE_SPLIT")) P.range_split = atoi(e);  // tuning knob (experiments)
   P.leaf_flat = 1;
   if (const char* e = getenv("TDFS_LEAF_FLAT")) P.leaf_flat = atoi(e);  // tuning knob (experiments)
@@ -1284,7 +1327,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     cudaEventRecord(ev0, st);
   }
   KernelFn fn = pick_kernel(mode, want_stats);
-  fn<<<L.blocks, L.wpb * 32, (size_t)L.wpb * L.fcap * sizeof(int), st>>>(P);
+  fn<<<L.blocks, L.wpb * 32, smem_bytes(L.wpb, L.fcap), st>>>(P);
   if ((e = cudaGetLastError()) != cudaSuccess) {
     cudaFree(d_trace);
     return cuda_fail(e, "kernel launch");

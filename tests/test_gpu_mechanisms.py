@@ -117,13 +117,15 @@ def test_split_counts_are_tau_invariant_on_skewed_graph():
             assert st["tasks_enqueued"] > 0 and st["tasks_enqueued"] == st["tasks_dequeued"]
 
 
-@pytest.mark.parametrize("range_split", ["1", "0"])
-def test_level2_range_tasks_k4(monkeypatch, range_split):
+@pytest.mark.parametrize("range_split,force", [("1", None), ("1", "1"), ("0", None)])
+def test_level2_range_tasks_k4(monkeypatch, range_split, force):
     """k = 4: a timed-out level-2 list is split into <= 32 id-range tasks <S0, S1, lo, hi>
      instead of one task per sibling.  With tau = 0 every level-2
     step splits; counts, per-level node counts and W (STATS variant) still equal the
     oracle's, and every pushed task is dequeued exactly once."""
     monkeypatch.setenv("TDFS_RANGE_SPLIT", range_split)
+    if force:  # range tasks also where the planner's heuristic prefers per-sibling tasks (k4)
+        monkeypatch.setenv("TDFS_RANGE_FORCE", force)
     g = T.rmat(11, 12, 4)
     for name in ("c4", "diamond", "k4", "tailed_triangle"):
         q = T.query(name)
