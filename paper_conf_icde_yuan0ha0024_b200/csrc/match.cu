@@ -605,9 +605,14 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   if (act && pl.lf_hi_var) hi = lane_lower_bound(F, lo, nF, x);
   if (!pl.lf_var) {
     long long cnt = (act && lo < hi) ? hi - lo : 0;
-    if (cnt && pl.lf_inj_var) {
-      const int i = lane_lower_bound(F, lo, hi, x);
-      cnt -= (i < hi && F[i] == x) ? 1 : 0;
+    if (cnt && pl.lf_inj_var) {  // x itself inside F[lo, hi)?
+      if (fr.hid >= 0) {            // referenced F of a hub y: range test + one bitmap load
+        cnt -= (x >= F[lo] && x <= F[hi - 1] &&
+                ((__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (x >> 5)) >> (x & 31)) & 1u)) ? 1 : 0;
+      } else {
+        const int i = lane_lower_bound(F, lo, hi, x);
+        cnt -= (i < hi && F[i] == x) ? 1 : 0;
+      }
     }
     for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
     return cnt;
