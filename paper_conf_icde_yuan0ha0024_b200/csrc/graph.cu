@@ -176,13 +176,14 @@ __global__ void hub_bits_kernel(const int64_t* __restrict__ offs, const int32_t*
 int build_hub_bitmaps(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs, std::vector<int32_t>& hub_vertices) {
   const long long words = (G.n + 31) / 32;
   if (G.n == 0 || words == 0) return TDFS_OK;
-  long long budget = 64ll << 20;
+  long long budget = 256ll << 20;  // measured on config 2: 16/64/256/1024 MB -> c4 2029/1416/1350/1350 ms
   if (const char* e = getenv("TDFS_HUB_BUDGET_MB")) budget = atoll(e) << 20;
   const long long max_hubs = budget / (words * 4);
   if (max_hubs <= 0) return TDFS_OK;
   cudaError_t e;
   std::vector<std::pair<int64_t, int32_t>> cand;
-  const int64_t min_deg = 256;
+  int64_t min_deg = 256;
+  if (const char* e = getenv("TDFS_HUB_MIN_DEG")) min_deg = std::max(1ll, atoll(e));  // tuning knob (experiments)
   for (int64_t v = 0; v < G.n; v++) {
     int64_t d = offs[v + 1] - offs[v];
     if (d >= min_deg) cand.push_back({-d, (int32_t)v});

@@ -447,7 +447,22 @@ struct FRef {
   int hid;       // by reference: y's bitmap row, -1 = none
   long long hb;  // by reference: y's hash set slots [hb, hb + hT)
   unsigned hT;   // 0 = none; hid < 0 && hT == 0 means F is materialised in shared memory
+  unsigned fix;  // by reference, plans without an N(S[k-2]) operand: lanes j whose S[j] must differ from
+                 // the leaf's candidates (injectivity at positions <= k-3) and lies inside F
 };
+
+// matched vertices S[j] (j in fr.fix) inside F[lo, hi): subtracted from a !lf_var leaf count
+// (warp-collective: every lane calls it, with its own window)
+__device__ __forceinline__ int fixed_in_window(const FRef& fr, int sreg, int lo, int hi) {
+  int n = 0;
+  const bool nonempty = lo < hi;
+  const int fmin = nonempty ? fr.F[lo] : 1, fmax = nonempty ? fr.F[hi - 1] : 0;
+  for (unsigned m = fr.fix; m; m &= m - 1) {
+    const int s = __shfl_sync(FULL, sreg, __ffs(m) - 1);
+    n += (s >= fmin && s <= fmax) ? 1 : 0;
+  }
+  return n;
+}
 
 // |{ v in L[s, e) : vmin <= v <= vmax, v in set }| for a sorted list L (global or shared
 // memory) and an O(1) probe set (bitmap row, else hash set).  Two 32-id batches per
@@ -509,7 +524,7 @@ __device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, const FRef& fr
   if (pl.lf_hi_var) hi = f_lower_bound(fr, lo, nF, x, lane);
   if (lo >= hi) return 0;
   if (!pl.lf_var) {
-    long long cnt = hi - lo;
+    long long cnt = hi - lo - fixed_in_window(fr, c.sreg, lo, hi);
     if (pl.lf_inj_var) {
       const int i = f_lower_bound(fr, lo, hi, x, lane);
       cnt -= (i < hi && F[i] == x) ? 1 : 0;
@@ -604,7 +619,8 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   if (act && pl.lf_lo_var) lo = lane_lower_bound(F, 0, nF, x + 1);
   if (act && pl.lf_hi_var) hi = lane_lower_bound(F, lo, nF, x);
   if (!pl.lf_var) {
-    long long cnt = (act && lo < hi) ? hi - lo : 0;
+    const int nfix = fr.fix ? fixed_in_window(fr, c.sreg, act ? lo : 0, act ? hi : 0) : 0;
+    long long cnt = (act && lo < hi) ? hi - lo - nfix : 0;
     if (cnt && pl.lf_inj_var) {  // x itself inside F[lo, hi)?
       if (fr.hid >= 0) {            // referenced F of a hub y: range test + one bitmap load
         cnt -= (x >= F[lo] && x <= F[hi - 1] &&
@@ -649,7 +665,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     pre[lane] = act ? p : tot;
     if (lane == 0) pre[32] = tot;
     __syncwarp();
-    int j = -1, jn = 0, pj = 0, lj = 0, hidj = -1, degj = 0;
+    int j = -1, jn = 0, pj = 0, lj = 0, hidj = -1, degj = 0, pb = 0;
     long long b0j = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
@@ -660,13 +676,15 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
           pj = pre[j];
           const LeafMeta e = meta[j];
           lj = e.lo; hidj = e.hid; degj = e.deg; b0j = e.b0;
+          pb = 0;
         }
         const int w = F[lj + idx - pj];
         if (hidj >= 0) {
           ok = (__ldg(P.hub_bits + (long long)hidj * P.hub_words + (w >> 5)) >> (w & 31)) & 1u;
         } else {
-          const int pos = lower_bound_dev(P.adj + b0j, degj, w);
-          ok = pos < degj && __ldg(P.adj + b0j + pos) == w;
+          // this lane's ids of one leaf increase round by round: search N(x_j) from the last hit
+          pb += lower_bound_dev(P.adj + b0j + pb, degj - pb, w);
+          ok = pb < degj && __ldg(P.adj + b0j + pb) == w;
         }
       }
       total += __popc(__ballot_sync(FULL, ok));
@@ -718,6 +736,7 @@ __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& 
   fr.hid = -1;
   fr.hb = 0;
   fr.hT = 0;
+  fr.fix = 0;
   if (pl.lf_byref && P.lf_byref) {
     const int y = getS(c.sreg, __ffs(pl.bwd[kVF]) - 1);
     const VMeta my = load_vmeta(P, y);
@@ -733,6 +752,17 @@ __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& 
       fr.hid = my.hid;
       fr.hb = my.hb;
       fr.hT = my.hT;
+      if (const uint32_t im = pl.inj_mask[kVF]) {  // matched S[j] (j <= k-3) that lie inside F
+        bool in = false;
+        if ((im >> lane) & 1u) {
+          const int s = c.sreg;
+          if (s >= wlo && s < whi) {
+            if (my.hid >= 0) in = (__ldg(P.hub_bits + (long long)my.hid * P.hub_words + (s >> 5)) >> (s & 31)) & 1u;
+            else in = hash_contains(P.hslots, my.hb, my.hT, s);
+          }
+        }
+        fr.fix = __ballot_sync(FULL, in);
+      }
       return (int)(b - a);
     }
   }

@@ -183,8 +183,10 @@ void build_dev(const QueryAdj& q, Plan& P) {
     d.lf_hi_var = (int8_t)((d.hi_mask[p] >> v) & 1u);
     d.lf_inj_var = (int8_t)((d.inj_mask[p] >> v) & 1u);
     d.lf_on = d.bwd[kVF] != 0;
+    // F referenced in place: one operand, no per-element filter; injectivity against positions
+    // <= k-3 only when the leaf count does not intersect N(S[k-2]) (then it is a subtraction)
     d.lf_byref = (int8_t)(__builtin_popcount(d.bwd[kVF]) == 1 && d.label[kVF] < 0 && d.deg_min[kVF] == 0 &&
-                          d.inj_mask[kVF] == 0);
+                          (d.inj_mask[kVF] == 0 || !d.lf_var));
     int best = -1;
     const int nb = __builtin_popcount(d.bwd[p]);
     for (int r = 2; r <= v; r++) {
