@@ -135,7 +135,7 @@ struct KParams {
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
   int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
-  int32_t smem_fcap;           // shared-memory layout: F ids per warp (the launch's, even when staging is off)
+  int32_t meta_off;            // shared-memory layout: byte offset of the warps' leaf-batch entries
   int32_t range_split;
   int32_t range_min, range_maxt;  // range tasks: >= range_min siblings each, <= range_maxt tasks per split
   int32_t range_mode;          // 0 auto (slice unless position 2's list is reused), 1 slice, 2 whole list

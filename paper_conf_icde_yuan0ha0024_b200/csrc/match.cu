@@ -59,6 +59,8 @@ __host__ __device__ inline size_t smem_bytes(int wpb, int fcap) {
   return smem_meta_offset(wpb, fcap) + (size_t)wpb * kMetaBytesPerWarp;
 }
 
+extern __shared__ __align__(16) int tdfs_smem[];  // [F stages of the block's warps][batch entries of the warps]
+
 // ------------------------------------------------------------ warp context
 template <bool STATS>
 struct Ctx {
@@ -71,8 +73,6 @@ struct Ctx {
   unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
   int* sF;                  // this warp's shared-memory stage for the leaf set F (P.fcap ints)
-  LeafMeta* sMeta;          // this warp's leaf-batch metadata (32 entries) ...
-  int* sPre;                // ... and the batch's exclusive prefix sums (33 ints)
   int w2lo, w2hi;           // range task: its level-2 candidates are the ids in [w2lo, w2hi) (warp-uniform)
   int w2mode;               // 0 no range task; 1 level 2 built as the slice only; 2 built whole, iterated in the slice
   int end2;                 // mode 2: iteration end index of level 2 (INT_MAX otherwise)
@@ -645,8 +645,10 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   }
   // the batch's per-leaf entries go to shared memory: a lane then reads its current leaf's
   // entry only when it moves to the next leaf (no warp-wide shuffles per element)
-  LeafMeta* meta = c.sMeta;
-  int* pre = c.sPre;
+  // shared-window addresses derived from tdfs_smem (32-bit LDS/STS, cheap to recompute)
+  char* const wbase = reinterpret_cast<char*>(tdfs_smem) + P.meta_off + (int)(threadIdx.x >> 5) * kMetaBytesPerWarp;
+  LeafMeta* meta = reinterpret_cast<LeafMeta*>(wbase);
+  int* pre = reinterpret_cast<int*>(wbase + 32 * sizeof(LeafMeta));
   if (act) {
     LeafMeta e;
     e.b0 = m.b0;
@@ -700,6 +702,44 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     __syncwarp();
     int j = -1, jn = 0, pj = 0, loj = 0, hij = 0, fminj = 0, fmaxj = 0;
     long long b0j = 0;
+#ifdef TDFS_B2
+    // two pairs per lane per round: both N(x) loads, then both probes, in flight together
+    for (int base = 0; base < tot; base += 64) {
+      int v[2], l2[2], h2[2];
+      bool in[2];
+#pragma unroll
+      for (int e = 0; e < 2; e++) {
+        const int idx = base + 32 * e + lane;
+        in[e] = idx < tot;
+        v[e] = 0;
+        if (in[e]) {
+          if (idx >= jn) {
+            do { ++j; jn = pre[j + 1]; } while (jn <= idx);
+            pj = pre[j];
+            const LeafMeta m2 = meta[j];
+            loj = m2.lo; hij = m2.hi; b0j = m2.b0;
+            fminj = F[loj];
+            fmaxj = F[hij - 1];
+          }
+          v[e] = __ldg(P.adj + b0j + idx - pj);
+          in[e] = v[e] >= fminj && v[e] <= fmaxj;
+          l2[e] = loj;
+          h2[e] = hij;
+        }
+      }
+      bool ok[2];
+#pragma unroll
+      for (int e = 0; e < 2; e++) {
+        ok[e] = false;
+        if (in[e]) {
+          if (fr.hid >= 0) ok[e] = (__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (v[e] >> 5)) >> (v[e] & 31)) & 1u;
+          else if (fr.hT) ok[e] = hash_contains(P.hslots, fr.hb, fr.hT, v[e]);
+          else ok[e] = F[smem_lower_bound(F, l2[e], h2[e], v[e])] == v[e];
+        }
+      }
+      total += __popc(__ballot_sync(FULL, ok[0])) + __popc(__ballot_sync(FULL, ok[1]));
+    }
+#else
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
       bool ok = false;
@@ -721,6 +761,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
       }
       total += __popc(__ballot_sync(FULL, ok));
     }
+#endif
   }
   __syncwarp();
   return total;
@@ -1015,14 +1056,7 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.w2mode = 0;
   c.end2 = INT_MAX;
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
-  extern __shared__ int smem_stage[];
-  c.sF = smem_stage + (threadIdx.x >> 5) * P.fcap;
-  {
-    char* meta = reinterpret_cast<char*>(smem_stage) + smem_meta_offset(blockDim.x >> 5, P.smem_fcap) +
-                 (threadIdx.x >> 5) * kMetaBytesPerWarp;
-    c.sMeta = reinterpret_cast<LeafMeta*>(meta);
-    c.sPre = reinterpret_cast<int*>(meta + 32 * sizeof(LeafMeta));
-  }
+  c.sF = tdfs_smem + (threadIdx.x >> 5) * P.fcap;
   const Queue q = make_queue(P);
   int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
   unsigned long long* cursor = ctr(P, C_CURSOR);
@@ -1301,7 +1335,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.E = L.E;
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
-  P.smem_fcap = L.fcap;
+  P.meta_off = (int)smem_meta_offset(L.wpb, L.fcap);
   P.lf_cost_g = 6;
   P.lf_cost_h = 2;
   if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
