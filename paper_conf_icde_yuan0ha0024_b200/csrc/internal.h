@@ -144,7 +144,8 @@ struct KParams {
   int32_t leaf_flat;           // staged leaves: flattened batch streams (else one leaf at a time)
   int32_t lf_byref;            // leaf staging: reference F in place when the plan allows (else materialise)
   int32_t lf_cost_g;
-  int32_t lf_cost_h;           // leaf staging cost model: extra cost of a hash probe over a bitmap probe           // leaf staging cost model: one dependent global load in shared-memory steps
+  int32_t lf_cost_h;
+  int32_t ua_hub, ub_ref;      // flat leaf batches: per-element cost of a bitmap probe in stream A / B           // leaf staging cost model: extra cost of a hash probe over a bitmap probe           // leaf staging cost model: one dependent global load in shared-memory steps
   int32_t coop_window;         // constraint windows by warp-cooperative 32-ary search (else per-lane binary)
   int32_t bsearch_variant;     // 0 halving, 1 power-of-two (experiments)
   // hub bitmaps (nullptr when off)

@@ -638,8 +638,8 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   int wA = 0, wB = 0;
   if (a > 0 && b > 0) {
     const int lgb = 32 - __clz(b), lga = 32 - __clz(a);
-    const long long uA = m.hid >= 0 ? 4 : 3 + lgb;
-    const long long uB = byref ? (fr.hid >= 0 ? 4 : 4 + P.lf_cost_h) : 3 + (lga >> 1);
+    const long long uA = m.hid >= 0 ? P.ua_hub : 3 + lgb;
+    const long long uB = byref ? (fr.hid >= 0 ? P.ub_ref : P.ub_ref + P.lf_cost_h) : 3 + (lga >> 1);
     if ((long long)a * uA <= (long long)b * uB) wA = a;
     else wB = b;
   }
@@ -702,44 +702,6 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     __syncwarp();
     int j = -1, jn = 0, pj = 0, loj = 0, hij = 0, fminj = 0, fmaxj = 0;
     long long b0j = 0;
-#ifdef TDFS_B2
-    // two pairs per lane per round: both N(x) loads, then both probes, in flight together
-    for (int base = 0; base < tot; base += 64) {
-      int v[2], l2[2], h2[2];
-      bool in[2];
-#pragma unroll
-      for (int e = 0; e < 2; e++) {
-        const int idx = base + 32 * e + lane;
-        in[e] = idx < tot;
-        v[e] = 0;
-        if (in[e]) {
-          if (idx >= jn) {
-            do { ++j; jn = pre[j + 1]; } while (jn <= idx);
-            pj = pre[j];
-            const LeafMeta m2 = meta[j];
-            loj = m2.lo; hij = m2.hi; b0j = m2.b0;
-            fminj = F[loj];
-            fmaxj = F[hij - 1];
-          }
-          v[e] = __ldg(P.adj + b0j + idx - pj);
-          in[e] = v[e] >= fminj && v[e] <= fmaxj;
-          l2[e] = loj;
-          h2[e] = hij;
-        }
-      }
-      bool ok[2];
-#pragma unroll
-      for (int e = 0; e < 2; e++) {
-        ok[e] = false;
-        if (in[e]) {
-          if (fr.hid >= 0) ok[e] = (__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (v[e] >> 5)) >> (v[e] & 31)) & 1u;
-          else if (fr.hT) ok[e] = hash_contains(P.hslots, fr.hb, fr.hT, v[e]);
-          else ok[e] = F[smem_lower_bound(F, l2[e], h2[e], v[e])] == v[e];
-        }
-      }
-      total += __popc(__ballot_sync(FULL, ok[0])) + __popc(__ballot_sync(FULL, ok[1]));
-    }
-#else
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
       bool ok = false;
@@ -761,7 +723,6 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
       }
       total += __popc(__ballot_sync(FULL, ok));
     }
-#endif
   }
   __syncwarp();
   return total;
@@ -1338,6 +1299,10 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.meta_off = (int)smem_meta_offset(L.wpb, L.fcap);
   P.lf_cost_g = 6;
   P.lf_cost_h = 2;
+  P.ua_hub = 4;
+  P.ub_ref = 4;
+  if (const char* e = getenv("TDFS_UA_HUB")) P.ua_hub = atoi(e);  // tuning knobs (experiments)
+  if (const char* e = getenv("TDFS_UB_REF")) P.ub_ref = atoi(e);
   if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
   P.range_split = 1;
   P.range_min = 32;
