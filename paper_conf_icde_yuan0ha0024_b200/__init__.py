@@ -46,6 +46,7 @@ TDFS_RUN_NO_SHORTCUT = 8
 TDFS_RUN_NO_HUB_BITMAP = 16
 TDFS_RUN_NO_LEAF_STAGE = 32
 TDFS_RUN_NO_HASH = 64
+TDFS_RUN_ARRAY_STACKS = 128
 TDFS_COUNT_INVALID = (1 << 64) - 1
 
 

@@ -1218,7 +1218,10 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   L->qcap = (uint64_t)(o->queue_ints / 3);
   L->qslots = 1;
   while (L->qslots < L->qcap) L->qslots <<= 1;
-  if (o->pool_bytes > 0) {
+  if (o->flags & TDFS_RUN_ARRAY_STACKS) {
+    // array-based stacks: every warp-level gets d_max ids (E whole pages) up front (Tables V/VII)
+    L->n_pages = (uint64_t)n_warps * L->n_levels * L->E;
+  } else if (o->pool_bytes > 0) {
     L->n_pages = (uint64_t)(o->pool_bytes / o->page_bytes);
   } else {
     // every warp-level able to reach d_max, capped at max(4 pages per warp-level, 2 GiB):
@@ -1294,6 +1297,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.n_pages = (uint32_t)L.n_pages;
   P.page_shift = L.page_shift;
   P.E = L.E;
+  P.array_stacks = (o->flags & TDFS_RUN_ARRAY_STACKS) ? 1 : 0;
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
   P.meta_off = (int)smem_meta_offset(L.wpb, L.fcap);
@@ -1352,7 +1356,11 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     init_queue_kernel<<<std::max(nb, 1), 256, 0, st>>>(P.slots, P.qslots, ticket_base);
   }
   size_t tbytes = sizeof(uint32_t) * (size_t)L.blocks * L.wpb * std::max(L.n_levels, 1) * L.E;
-  if (L.n_levels > 0) cudaMemsetAsync(P.page_tables, 0xff, tbytes, st);
+  if (L.n_levels > 0 && !P.array_stacks) cudaMemsetAsync(P.page_tables, 0xff, tbytes, st);
+  if (L.n_levels > 0 && P.array_stacks) {  // all pages owned up front: the pool cursor starts exhausted
+    const unsigned long long np = L.n_pages;
+    cudaMemcpyAsync(P.ctr + C_POOL * kCounterStride, &np, sizeof(np), cudaMemcpyHostToDevice, st);
+  }
 
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   if (want_stats) {

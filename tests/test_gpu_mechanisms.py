@@ -139,3 +139,19 @@ def test_level2_range_tasks_k4(monkeypatch, range_split, force):
             assert st["tasks_enqueued"] == st["tasks_dequeued"], (name, kw)
             assert U.count(g, q, "auto", order=order, **kw) == r["count"], (name, kw)
         assert st["tasks_enqueued"] > 0
+
+
+def test_array_stacks_ablation_same_results():
+    """NEXT-4 / E10: array-based stacks (every warp-level owns d_max ids up front, the paper's
+    baseline of Tables V-VIII) give the same counts and node counts as paged stacks, and
+    their pool is exactly n_warps x levels x E pages."""
+    g = T.rmat(11, 12, 4)
+    for name in ("c4", "diamond", "house", "c5", "prism"):
+        q = T.query(name)
+        ref = O.count(g, q, "auto", threads=8)
+        for kw in (dict(), dict(tau_ms=0.0), dict(page_bytes=128)):
+            cnt, st = U.count(g, q, "auto", stats=True, flags=M.TDFS_RUN_ARRAY_STACKS, **kw)
+            assert cnt == ref, (name, kw)
+            assert st["pages_used"] == st["pool_pages"] == (
+                st["grid_blocks"] * st["warps_per_block"] * (q.k - 3) * st["page_table_entries"]), (name, kw)
+            assert U.count(g, q, "auto", flags=M.TDFS_RUN_ARRAY_STACKS, **kw) == ref
