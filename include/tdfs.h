@@ -146,7 +146,7 @@ void tdfs_free_plan(tdfs_plan* p);
 #define TDFS_RUN_NO_HUB_BITMAP 16u  /* ablation: probe hub adjacency lists by search, not by bitmap */
 #define TDFS_RUN_NO_LEAF_STAGE 32u  /* ablation: no shared-memory staging of the last position's fixed part */
 #define TDFS_RUN_NO_HASH 64u        /* ablation: probe non-hub adjacency lists by binary search, not by the hash index */
-#define TDFS_RUN_ARRAY_STACKS 128u  /* ablation: array-based stacks (d_max ids per warp-level up front, Tables V-VIII) instead of pages */
+#define TDFS_RUN_ARRAY_STACKS 128u  /* ablation: array-based stack memory (d_max ids per warp-level up front, identity page tables: no page is ever allocated; Tables V-VIII) */
 
 typedef struct {
   int64_t tau_ns;              /* timeout tau; default 10 ms;

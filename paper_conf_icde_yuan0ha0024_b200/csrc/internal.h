@@ -131,7 +131,7 @@ struct KParams {
   uint32_t n_pages;
   int32_t page_shift;          // log2(ints per page)
   int32_t E;                   // page-table entries per level
-  int32_t array_stacks;        // ablation: contiguous per-warp-level arrays of E pages, no page table
+  int32_t array_stacks;        // ablation: contiguous per-warp-level arrays of E pages (identity page tables)
   int64_t tau_ns;              // < 0: infinity
   int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
   int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)

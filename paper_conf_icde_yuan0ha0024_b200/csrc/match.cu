@@ -1133,6 +1133,12 @@ __global__ void init_queue_kernel(QSlot* slots, unsigned long long cap, unsigned
   }
 }
 
+__global__ void iota_u32_kernel(uint32_t* a, unsigned long long n) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    a[i] = (uint32_t)i;
+}
+
 __global__ void init_counters_kernel(unsigned long long* ctrs, unsigned long long qcap, unsigned long long base) {
   int i = threadIdx.x;
   if (i < C_NUM * kCounterStride) ctrs[i] = 0;
@@ -1357,7 +1363,11 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   }
   size_t tbytes = sizeof(uint32_t) * (size_t)L.blocks * L.wpb * std::max(L.n_levels, 1) * L.E;
   if (L.n_levels > 0 && !P.array_stacks) cudaMemsetAsync(P.page_tables, 0xff, tbytes, st);
-  if (L.n_levels > 0 && P.array_stacks) {  // all pages owned up front: the pool cursor starts exhausted
+  if (L.n_levels > 0 && P.array_stacks) {
+    // array layout: warp-level t owns pages [t*E, (t+1)*E) up front (identity page tables), so no page is
+    // ever allocated or found missing during the job; the pool cursor starts exhausted
+    const uint64_t nt = (uint64_t)L.blocks * L.wpb * L.n_levels * L.E;
+    iota_u32_kernel<<<(int)std::min<uint64_t>((nt + 255) / 256, 65535), 256, 0, st>>>(P.page_tables, nt);
     const unsigned long long np = L.n_pages;
     cudaMemcpyAsync(P.ctr + C_POOL * kCounterStride, &np, sizeof(np), cudaMemcpyHostToDevice, st);
   }

@@ -226,9 +226,6 @@ __device__ __forceinline__ uint32_t ensure_page(const KParams& P, uint32_t* tabl
 
 // Paged reader (the [] operator of Alg. 5 for reads): element pos of a level.
 __device__ __forceinline__ int32_t paged_read(const KParams& P, const uint32_t* table, long long pos) {
-  // array-stack ablation (TDFS_RUN_ARRAY_STACKS, the paper's "array-based" baseline, Tables V-VIII):
-  // every warp-level owns E contiguous pages, addressed directly without the page table
-  if (P.array_stacks) return P.pool[((long long)(table - P.page_tables) << P.page_shift) + pos];
   uint32_t pg = table[pos >> P.page_shift];
   return page_base(P, pg)[pos & ((1ll << P.page_shift) - 1)];
 }
@@ -247,12 +244,6 @@ __device__ __forceinline__ bool paged_write(const KParams& P, PagedWriter& w, un
   int cnt = __popc(ballot);
   if (cnt == 0) return true;
   const int shift = P.page_shift;
-  if (P.array_stacks) {
-    if (pos0 + cnt > ((long long)P.E << shift)) return false;
-    if (ballot >> lane & 1u)
-      P.pool[((long long)(w.table - P.page_tables) << shift) + pos0 + __popc(ballot & lanemask_lt())] = v;
-    return true;
-  }
   int pf = (int)(pos0 >> shift);
   int pl = (int)((pos0 + cnt - 1) >> shift);
   uint32_t pgf = w.cur_pg, pgl = w.cur_pg;

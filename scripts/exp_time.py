@@ -28,7 +28,12 @@ for name in qn:
                 k, v = kv.split("=")
                 saved[k] = os.environ.get(k)
                 os.environ[k] = v
-        o = M.default_opts(flags=int(fl or 0), shard_world=W)
+        kw = {}
+        for kv in os.environ.get("EXP_OPTS", "").split(","):  # e.g. EXP_OPTS=chunk=32,tau_ms=1
+            if kv:
+                k, v = kv.split("=")
+                kw[k] = float(v) if "." in v else int(v)
+        o = M.default_opts(flags=int(fl or 0), shard_world=W, **kw)
         ts = []
         for r in range(reps + 1):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
