@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--tau-ms", type=float, default=10.0)
+    ap.add_argument("--chunk", type=int, default=1,
+                    help="initial edge tasks per cursor grab (ABI default 8 = the paper's; 1 measured best on config 2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--queries", type=str, default="")
@@ -214,7 +216,8 @@ def run_ours(a):
     plans = [M.plan_from_query(q) for q in qs]
     plan_s = time.perf_counter() - t_plan0
     tau = None if a.tau_ms < 0 else a.tau_ms
-    opts = M.default_opts(tau_ms=tau, shard_rank=rank, shard_world=world * a.profile_shard_world, flags=a.flags)
+    opts = M.default_opts(tau_ms=tau, chunk=a.chunk, shard_rank=rank, shard_world=world * a.profile_shard_world,
+                          flags=a.flags)
     ws_bytes = max(M.tdfs_workspace_bytes(h, p, opts) for p in plans)
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
     d_counts = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
@@ -350,7 +353,7 @@ def run_ours(a):
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"config{a.config}: {desc}", "n": g.n, "m": info["m"], "dmax": info["dmax"],
                        "queries": [q.name for q in qs], "constraints": "full symmetry breaking (stabilizer chain)",
-                       "tau_ms": a.tau_ms, "parallelism": f"shard{world}",
+                       "tau_ms": a.tau_ms, "chunk": a.chunk, "parallelism": f"shard{world}",
                        "l2": "flushed (256 MB write) before every timed step", "load_s": load_s, "plan_s": plan_s,
                        "per_query": per_query},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
