@@ -216,9 +216,11 @@ def run_ours(a):
     plans = [M.plan_from_query(q) for q in qs]
     plan_s = time.perf_counter() - t_plan0
     tau = None if a.tau_ms < 0 else a.tau_ms
-    opts = M.default_opts(tau_ms=tau, chunk=a.chunk, shard_rank=rank, shard_world=world * a.profile_shard_world,
-                          flags=a.flags)
-    ws_bytes = max(M.tdfs_workspace_bytes(h, p, opts) for p in plans)
+    # per query: k = 3 jobs are one intersection per edge task, so they keep the paper's chunk of 8
+    # (one cursor atomic per edge costs the triangle 4.8 -> 17.4 ms); deeper queries take a.chunk
+    qopts = [M.default_opts(tau_ms=tau, chunk=(8 if q.k <= 3 else a.chunk), shard_rank=rank,
+                            shard_world=world * a.profile_shard_world, flags=a.flags) for q in qs]
+    ws_bytes = max(M.tdfs_workspace_bytes(h, p, o) for p, o in zip(plans, qopts))
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
     d_counts = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{dev}")
@@ -226,7 +228,7 @@ def run_ours(a):
     # W (algorithmic adjacency bytes) per query from one instrumented run (untimed)
     W, Wfull, stats_runs = [], [], []
     for p in plans:
-        c, st = M.tdfs_count(h, p, opts, workspace=ws, stats=True)
+        c, st = M.tdfs_count(h, p, qopts[len(W)], workspace=ws, stats=True)
         W.append(st["stream_bytes"])   # roofline bytes, R29b
         Wfull.append(st["adj_bytes"])  # SURVEY 8(d) full-operand W, for reference
         stats_runs.append(st)
@@ -235,7 +237,7 @@ def run_ours(a):
         for i, p in enumerate(plans):
             if ev_q is not None:
                 ev_q[i][0].record(stream)
-            M.tdfs_count(h, p, opts, workspace=ws, stream=stream, d_count=d_counts[i:i + 1], sync=False)
+            M.tdfs_count(h, p, qopts[i], workspace=ws, stream=stream, d_count=d_counts[i:i + 1], sync=False)
             if ev_q is not None:
                 ev_q[i][1].record(stream)
         if world > 1:
@@ -315,7 +317,7 @@ def run_ours(a):
             tot = 0
             dc = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
             for i, p in enumerate(pl):
-                M.tdfs_count(hh, p, opts, workspace=ws, stream=stream, d_count=dc[i:i + 1], sync=False)
+                M.tdfs_count(hh, p, qopts[i], workspace=ws, stream=stream, d_count=dc[i:i + 1], sync=False)
             if world > 1:
                 dist.all_reduce(dc)
             tot = int(dc.cpu().sum().item())
@@ -353,7 +355,7 @@ def run_ours(a):
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"config{a.config}: {desc}", "n": g.n, "m": info["m"], "dmax": info["dmax"],
                        "queries": [q.name for q in qs], "constraints": "full symmetry breaking (stabilizer chain)",
-                       "tau_ms": a.tau_ms, "chunk": a.chunk, "parallelism": f"shard{world}",
+                       "tau_ms": a.tau_ms, "chunk": {"k3": 8, "k>=4": a.chunk}, "parallelism": f"shard{world}",
                        "l2": "flushed (256 MB write) before every timed step", "load_s": load_s, "plan_s": plan_s,
                        "per_query": per_query},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
