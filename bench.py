@@ -10,8 +10,14 @@ diamond, tailed triangle and 4-clique, each counted once per step with full symm
 breaking.  A step = the five tdfs_count jobs (one persistent kernel each).  Inputs are
 resident in HBM before timing; L2 (126 MB) is flushed before every timed step because
 the CSR (~32 MB) would otherwise stay cached across steps.
-N > 1 (torchrun): every rank counts its round-robin shard of the directed initial edges
- and one NCCL all-reduce sums the counts -- total work is fixed: "strong".
+N > 1 (torchrun): every rank counts its shard of the directed initial edges (round-robin,
+PAPER.md:522, or --shard-policy 1 degree-balanced, R31; or --shared-cursor: all ranks
+take edge chunks from one cursor in rank 0's HBM, NEXT-3) and one NCCL all-reduce of
+{count, failed} sums the counts -- total work is fixed: "strong".
+
+After timing, the counts are checked against the oracle goldens of the config
+(tests/golden/c<cfg>_counts.txt, written by scripts/golden_counts.py from oracle/ only) when
+the file has them; a mismatch or a failed job (TDFS_COUNT_INVALID) aborts the run.
 
 Prints ONE JSON line (rank 0).
 """
@@ -50,6 +56,9 @@ def parse():
     ap.add_argument("--profile-shard-world", type=int, default=1,
                     help="profiling only: run shard 0 of W on one GPU (not a bench number)")
     ap.add_argument("--flags", type=int, default=0, help="tdfs_run_opts.flags (ablations)")
+    ap.add_argument("--shard-policy", type=int, default=0, help="N > 1: 0 round-robin (paper), 1 degree-balanced")
+    ap.add_argument("--shared-cursor", action="store_true", help="N > 1: cross-GPU shared chunk cursor (NEXT-3)")
+    ap.add_argument("--hub-bitmap-mb", type=int, default=0, help="hub bitmap budget (0 = library default)")
     return ap.parse_args()
 
 
@@ -124,31 +133,76 @@ def measured_peaks():
     return 6650.0, "fallback"
 
 
-def ncu_traffic(cfg: int):
-    """dram bytes per launch of the matching kernel from the committed ncu --set full summary."""
+def kernel_source_hash() -> str:
+    """sha256 of the product's CUDA/C++ sources: ties a committed ncu summary to the kernel build."""
+    import hashlib
+    h = hashlib.sha256()
+    csrc = os.path.join(ROOT, "paper_conf_icde_yuan0ha0024_b200", "csrc")
+    for f in sorted(os.listdir(csrc)) + ["../../include/tdfs.h"]:
+        with open(os.path.join(csrc, f), "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()[:16]
+
+
+def ncu_summary(cfg: int):
+    """Per-query ncu --set full numbers of THIS kernel build (profiles/ncu_full_summary.json,
+    written by scripts/ncu_summary.py with the source hash); None when the build differs."""
     p = os.path.join(ROOT, "profiles", "ncu_full_summary.json")
     if not os.path.exists(p):
         return None
     with open(p) as f:
         d = json.load(f)
-    return d.get("dram_bytes_per_launch")
+    if d.get("source_hash") != kernel_source_hash() or d.get("config") != cfg:
+        return None
+    return d
+
+
+def goldens(cfg: int):
+    p = os.path.join(ROOT, "tests", "golden", f"c{cfg}_counts.txt")
+    out = {}
+    if os.path.exists(p):
+        for line in open(p):
+            if line.strip() and not line.startswith("#"):
+                k, v = line.split(":", 1)
+                out[k.strip()] = int(v.split()[0])
+    return out
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def cpu_baseline(g, qs, sample_world: int):
     """The oracle (as it stands) on a bounded sample: 1/sample_world of the directed root
-    edges of every query, all host cores."""
+    edges of every query, all host cores; plus the single-threaded oracle on 1/(10 W)."""
     import oracle as O
     threads = os.cpu_count() or 1
+    og = O.OracleGraph(g)
     tot_m, tot_t = 0, 0.0
     for q in qs:
         t0 = time.perf_counter()
-        c = O.count(g, q, "auto", shard=(0, sample_world), threads=threads)
+        c = O.count(og, q, "auto", shard=(0, sample_world), threads=threads)
         tot_t += time.perf_counter() - t0
         tot_m += c
+    w1 = 10 * sample_world + 1
+    one_m, one_t = 0, 0.0
+    for q in qs:
+        t0 = time.perf_counter()
+        one_m += O.count(og, q, "auto", shard=(0, w1), threads=1)
+        one_t += time.perf_counter() - t0
     return {"value": tot_m / tot_t if tot_t > 0 else 0.0, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "cpu_model": cpu_model(),
+            "single_core_value": one_m / one_t if one_t > 0 else 0.0,
             "sample": f"each query on the directed root edges with rank = 0 mod {sample_world} "
                       f"(1/{sample_world} of the initial tasks), serial Alg. 1 fanned out over roots; "
-                      f"{tot_m} matches in {tot_t:.2f} s incl. adjacency build"}
+                      f"{tot_m} matches in {tot_t:.2f} s; single core: 1/{w1} of the root edges, "
+                      f"{one_m} matches in {one_t:.2f} s"}
 
 
 # ------------------------------------------------------------------ reference arm
@@ -207,8 +261,9 @@ def run_ours(a):
     if a.queries:
         keep = set(a.queries.split(","))
         qs = [q for q in qs if q.name in keep or q.name.replace("_lab", "") in keep]
+    hub_bytes = a.hub_bitmap_mb << 20
     t_load0 = time.perf_counter()
-    h = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev)
+    h = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes)
     torch.cuda.synchronize()
     load_s = time.perf_counter() - t_load0
     info = h.info()
@@ -216,32 +271,45 @@ def run_ours(a):
     plans = [M.plan_from_query(q) for q in qs]
     plan_s = time.perf_counter() - t_plan0
     tau = None if a.tau_ms < 0 else a.tau_ms
+    cursors = D.SharedCursorGroup(dev) if (world > 1 and a.shared_cursor) else None
     # per query: k = 3 jobs are one intersection per edge task, so they keep the paper's chunk of 8
     # (one cursor atomic per edge costs the triangle 4.8 -> 17.4 ms); deeper queries take a.chunk
     qopts = [M.default_opts(tau_ms=tau, chunk=(8 if q.k <= 3 else a.chunk), shard_rank=rank,
-                            shard_world=world * a.profile_shard_world, flags=a.flags) for q in qs]
+                            shard_world=world * a.profile_shard_world, shard_policy=a.shard_policy,
+                            flags=a.flags) for q in qs]
+    if cursors is not None:
+        for o in qopts:
+            o.shared_cursor = cursors.cursor.ptr
     ws_bytes = max(M.tdfs_workspace_bytes(h, p, o) for p, o in zip(plans, qopts))
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
     d_counts = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{dev}")
 
-    # W (algorithmic adjacency bytes) per query from one instrumented run (untimed)
+    # roofline bytes (R32) and W per query from one instrumented run (untimed;
+    # with a shared cursor the STATS run takes this rank's static shard instead)
     W, Wfull, stats_runs = [], [], []
-    for p in plans:
-        c, st = M.tdfs_count(h, p, qopts[len(W)], workspace=ws, stats=True)
-        W.append(st["stream_bytes"])   # roofline bytes, R29b
-        Wfull.append(st["adj_bytes"])  # SURVEY 8(d) full-operand W, for reference
+    for p, o in zip(plans, qopts):
+        so = M.tdfs_run_opts.from_buffer_copy(o)
+        so.shared_cursor = None
+        c, st = M.tdfs_count(h, p, so, workspace=ws, stats=True)
+        W.append(st["stream_bytes"])
+        Wfull.append(st["adj_bytes"])
         stats_runs.append(st)
 
+    def launch(i, ev_q=None):
+        if ev_q is not None:
+            ev_q[i][0].record(stream)
+        M.tdfs_count(h, plans[i], qopts[i], workspace=ws, stream=stream, d_count=d_counts[i:i + 1], sync=False)
+        if ev_q is not None:
+            ev_q[i][1].record(stream)
+
     def step(ev_q=None):
-        for i, p in enumerate(plans):
-            if ev_q is not None:
-                ev_q[i][0].record(stream)
-            M.tdfs_count(h, p, qopts[i], workspace=ws, stream=stream, d_count=d_counts[i:i + 1], sync=False)
-            if ev_q is not None:
-                ev_q[i][1].record(stream)
-        if world > 1:
-            dist.all_reduce(d_counts)
+        for i in range(len(plans)):
+            if cursors is not None:
+                cursors.prepare(stream)  # zero the shared cursor, fence all ranks (host sync)
+            launch(i, ev_q)
+            if cursors is not None:
+                cursors.finish()
 
     for _ in range(a.warmup):
         flush.zero_()
@@ -264,38 +332,62 @@ def run_ours(a):
             dist.barrier()
         ev0.record(stream)
         step(evq)
+        if world > 1:  # the one exchange: {count, failed} per query (checked)
+            summed = D.reduce_counts(d_counts.clone())
         ev1.record(stream)
         torch.cuda.synchronize()
         step_ms.append(ev0.elapsed_time(ev1))
         for i, (e0, e1) in enumerate(evq):
             q_ms[i].append(e0.elapsed_time(e1))
-        counts = d_counts.cpu().tolist()
+        local_counts = d_counts.cpu().tolist()
+        if any(c == D.COUNT_INVALID_I64 for c in local_counts):  # a failed job is an error, never a count
+            raise RuntimeError(f"tdfs job failed (TDFS_COUNT_INVALID) in step {s}: {local_counts}")
+        counts = summed.cpu().tolist() if world > 1 else local_counts
     clk = clocks.stop()
     M.tdfs_workspace_status(ws, stream, dev)
 
     total_ms = sum(step_ms)
+    q_med = [statistics.median(x) for x in q_ms]
     if world > 1:
-        t = torch.tensor([total_ms], dtype=torch.float64, device=f"cuda:{dev}")
+        t = torch.tensor([total_ms] + [sum(x) for x in q_ms] + q_med, dtype=torch.float64, device=f"cuda:{dev}")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
-        qt = torch.tensor([sum(x) for x in q_ms], dtype=torch.float64, device=f"cuda:{dev}")
-        dist.all_reduce(qt, op=dist.ReduceOp.MAX)
-        q_tot = qt.tolist()
+        tl = t.tolist()
+        total_ms, q_tot, q_med = tl[0], tl[1:1 + len(qs)], tl[1 + len(qs):]
     else:
         q_tot = [sum(x) for x in q_ms]
     matches_per_step = int(sum(counts))
     value = matches_per_step * a.steps / (total_ms / 1000.0)
 
-    # roofline of the dominant kernel (the matching kernel; 1 launch per query per step)
+    # parity: every full count equals the oracle golden of this config (when present)
+    gold = goldens(a.config) if a.profile_shard_world == 1 else {}  # counts are full counts (all-reduced)
+    parity = {}
+    for i, q in enumerate(qs):
+        gname = q.name.replace("_lab", "")
+        if gname in gold:
+            if counts[i] != gold[gname]:
+                raise RuntimeError(f"count mismatch vs oracle golden for {gname}: {counts[i]} != {gold[gname]}")
+            parity[gname] = "equal to oracle golden"
+
+    # roofline of the dominant kernel: the matching launch of the slowest query (one launch per
+    # query per step); achieved = its R32 bytes per launch / its mean launch time (CUDA events)
     peak, peak_kind = measured_peaks()
-    w_local = sum(W)  # this rank's shard bytes per step
-    per_launch_bytes = w_local / len(qs)
-    avg_launch_s = (sum(q_tot) / len(qs)) / a.steps / 1000.0
-    achieved = per_launch_bytes / avg_launch_s / 1e9
-    traffic = ncu_traffic(a.config)
+    dom = max(range(len(qs)), key=lambda i: q_tot[i])
+    dom_s = q_tot[dom] / a.steps / 1000.0
+    achieved = W[dom] / dom_s / 1e9
+    ncu = ncu_summary(a.config)
+    traffic, l2 = None, None
+    if ncu is not None and qs[dom].name in ncu.get("per_query", {}):
+        nq = ncu["per_query"][qs[dom].name]
+        traffic = nq.get("dram_bytes")
+        if nq.get("lts_bytes") is not None:
+            l2 = {"lts_t_bytes": nq["lts_bytes"], "ncu_duration_ms": nq.get("duration_ms"),
+                  "achieved_GBps": nq["lts_bytes"] / (nq["duration_ms"] / 1000.0) / 1e9,
+                  "peak_GBps": ncu.get("l2_peak_gbs"), "l2_hit_rate": nq.get("l2_hit"),
+                  "frac": (nq["lts_bytes"] / (nq["duration_ms"] / 1000.0) / 1e9) / ncu["l2_peak_gbs"]
+                  if ncu.get("l2_peak_gbs") else None}
 
     # e2e through the public API with host buffers: H2D of the CSR from pinned memory,
-    # load, plan, the five counts, D2H of the counts -- every step
+    # load, plan, the counts, D2H of the counts -- every step
     e2e = None
     if not a.no_e2e:
         import tdfs_inputs as T
@@ -312,19 +404,22 @@ def run_ours(a):
                 dist.barrier()
             t0 = time.perf_counter()
             hh = M.tdfs_load_graph(offs_h.numpy(), adj_h.numpy(), None if lab_h is None else lab_h.numpy(),
-                                   device=dev)
+                                   device=dev, hub_bitmap_bytes=hub_bytes)
             pl = [M.plan_from_query(q) for q in qs]
-            tot = 0
             dc = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
             for i, p in enumerate(pl):
+                if cursors is not None:
+                    cursors.prepare(stream)
                 M.tdfs_count(hh, p, qopts[i], workspace=ws, stream=stream, d_count=dc[i:i + 1], sync=False)
-            if world > 1:
-                dist.all_reduce(dc)
-            tot = int(dc.cpu().sum().item())
+                if cursors is not None:
+                    cursors.finish()
+            tot = D.reduce_counts(dc)  # checked (and all-reduced for N > 1)
+            tot = int(tot.sum().item())
             dt = time.perf_counter() - t0
             hh.free()
             if s >= a.warmup:
                 e2e_t.append(dt)
+            assert tot == matches_per_step, (tot, matches_per_step)
         et = sum(e2e_t)
         if world > 1:
             t = torch.tensor([et], dtype=torch.float64, device=f"cuda:{dev}")
@@ -332,8 +427,8 @@ def run_ours(a):
             et = float(t.item())
         e2e = {"value": matches_per_step * a.steps / et, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": 8 * len(qs),
-               "includes": "tdfs_load_graph (H2D of pinned CSR, src build), tdfs_plan_query x5, tdfs_count x5, "
-                           "D2H of the counts"}
+               "includes": f"tdfs_load_graph (H2D of pinned CSR, src array, hub bitmaps), tdfs_plan_query x{len(qs)}, "
+                           f"tdfs_count x{len(qs)}, checked reduce + D2H of the counts"}
 
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
@@ -342,35 +437,44 @@ def run_ours(a):
     if rank == 0:
         per_query = {}
         for i, q in enumerate(qs):
+            t_s = q_tot[i] / a.steps / 1000.0
             per_query[q.name] = {"count": int(counts[i]), "time_to_count_ms": q_tot[i] / a.steps,
-                                 "matches_per_s": counts[i] / (q_tot[i] / a.steps / 1000.0),
-                                 "W_bytes": int(W[i]), "W_full_bytes": int(Wfull[i]),
-                                 "eff_GBps": W[i] / (q_tot[i] / a.steps / 1000.0) / 1e9,
+                                 "time_to_count_median_ms": q_med[i],
+                                 "matches_per_s": counts[i] / t_s,
+                                 "roofline_bytes": int(W[i]), "W_full_bytes": int(Wfull[i]),
+                                 "eff_GBps": W[i] / t_s / 1e9, "frac": W[i] / t_s / 1e9 / peak,
                                  "timeouts": int(stats_runs[i]["timeouts"]),
                                  "tasks_enqueued": int(stats_runs[i]["tasks_enqueued"]),
-                                 "pages_used": int(stats_runs[i]["pages_used"])}
+                                 "pages_used": int(stats_runs[i]["pages_used"]),
+                                 "nodes_per_level": stats_runs[i]["nodes_per_level"][:q.k]}
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
             "ms_per_step": total_ms / a.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"config{a.config}: {desc}", "n": g.n, "m": info["m"], "dmax": info["dmax"],
                        "queries": [q.name for q in qs], "constraints": "full symmetry breaking (stabilizer chain)",
-                       "tau_ms": a.tau_ms, "chunk": {"k3": 8, "k>=4": a.chunk}, "parallelism": f"shard{world}",
+                       "tau_ms": a.tau_ms, "chunk": {"k3": 8, "k>=4": a.chunk},
+                       "parallelism": f"shard{world}" + ("-shared-cursor" if cursors is not None else
+                                                         f"-policy{a.shard_policy}"),
                        "l2": "flushed (256 MB write) before every timed step", "load_s": load_s, "plan_s": plan_s,
-                       "per_query": per_query},
+                       "parity": parity or "no goldens for this config / shard", "per_query": per_query},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "peak_kind": peak_kind,
-                         "note": "achieved = algorithmic bytes per matching-kernel launch (DESIGN.md R29b: 16 B per "
-                                 "Eq.(1) operand + 4 B x smallest constraint-windowed operand, per extension; from one "
-                                 "STATS run) / mean tdfs_count duration (CUDA events on the launch stream); traffic = "
-                                 "ncu dram bytes per launch (profiles/ncu_full_summary.json)"},
+                         "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                         "kernel": f"tdfs_kernel<0,0> ({qs[dom].name}, the dominant launch)",
+                         "l2": l2,
+                         "note": "achieved = algorithmic bytes of the dominant matching launch (DESIGN.md R32: per "
+                                 "extension 16 B per Eq.(1) operand + 4 B x the smallest constraint-windowed Eq.(1) "
+                                 "source, 0 for a count-only last position; one STATS run) / its mean tdfs_count "
+                                 "duration (CUDA events on the launch stream); traffic = ncu dram bytes of that "
+                                 "launch from profiles/ncu_full_summary.json of this source hash (else null)"},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": 4 * len(qs) * a.steps,
             "clocks": clk,
         }
         print(json.dumps(line), flush=True)
+    if cursors is not None:
+        cursors.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()

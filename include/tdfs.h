@@ -36,7 +36,7 @@
 extern "C" {
 #endif
 
-#define TDFS_ABI_VERSION 1
+#define TDFS_ABI_VERSION 2
 #define TDFS_MAX_K 8
 
 typedef enum {
@@ -83,18 +83,22 @@ typedef struct {
   const uint8_t* label;  /* [n] or NULL (unlabeled: every label is 0) */
   int32_t mem;           /* TDFS_MEM_HOST_COPY or TDFS_MEM_DEVICE_BORROW */
   uint32_t flags;        /* TDFS_GRAPH_VALIDATE | TDFS_GRAPH_NORMALIZE */
+  int64_t hub_bitmap_bytes; /* device bytes for hub adjacency bitmaps (n bits per hub, vertices of degree
+                               >= 256, highest degree first): 0 = default 256 MB, < 0 = none */
 } tdfs_csr;
 
 /* Load a CSR graph onto CUDA device `device`.  Uploads (HOST_COPY) or borrows the
  * arrays, computes d_max and the per-entry source array used by the edge tasks
- * (PAPER.md:120-122).  Errors: INVALID_ARG, GRAPH_FORMAT, ID_RANGE, OOM, CUDA. */
+ * (PAPER.md:120-122), builds the hub bitmaps.  Without VALIDATE the offsets and the
+ * id range [0, n) are still checked (cheaply).  Errors: INVALID_ARG, GRAPH_FORMAT,
+ * ID_RANGE, OOM, CUDA. */
 int tdfs_load_graph(const tdfs_csr* g, int device, void* stream, tdfs_graph** out);
 
 /* Load from an undirected edge list (host arrays, m pairs; any orientation,
  * duplicates and self-loops allowed -- they are normalised away on the host with
  * multiple threads).  label: host [n] or NULL. */
 int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const int32_t* dst, const uint8_t* label,
-                    int device, void* stream, tdfs_graph** out);
+                    int64_t hub_bitmap_bytes /* as in tdfs_csr */, int device, void* stream, tdfs_graph** out);
 
 /* n, undirected edge count m = nnz/2, maximum degree, number of labels (max+1, 1 if unlabeled). */
 int tdfs_graph_info(const tdfs_graph* g, int64_t* n, int64_t* m, int64_t* dmax, int32_t* nlabels);
@@ -145,8 +149,14 @@ void tdfs_free_plan(tdfs_plan* p);
 #define TDFS_RUN_NO_SHORTCUT 8u     /* ablation: always scan the last level (no count-only window shortcut) */
 #define TDFS_RUN_NO_HUB_BITMAP 16u  /* ablation: probe hub adjacency lists by search, not by bitmap */
 #define TDFS_RUN_NO_LEAF_STAGE 32u  /* ablation: no shared-memory staging of the last position's fixed part */
-#define TDFS_RUN_NO_HASH 64u        /* ablation: probe non-hub adjacency lists by binary search, not by the hash index */
 #define TDFS_RUN_ARRAY_STACKS 128u  /* ablation: array-based stack memory (d_max ids per warp-level up front, identity page tables: no page is ever allocated; Tables V-VIII) */
+#define TDFS_RUN_NO_RANGE_TASKS 256u /* ablation: k = 4 timeout splits push one task per sibling instead of id-range tasks (R30) */
+
+/* Partition of the initial edge tasks over shard_world ranks. */
+#define TDFS_SHARD_ROUND_ROBIN 0      /* directed edge e (CSR index) -> rank e mod W */
+#define TDFS_SHARD_DEGREE_BALANCED 1  /* heavy roots (cost = sum of neighbour degrees > total/(64 W)) dealt by
+                                         edge round-robin; the other roots dealt whole in snake order of
+                                         decreasing cost (R31) */
 
 typedef struct {
   int64_t tau_ns;              /* timeout tau; default 10 ms;
@@ -158,9 +168,17 @@ typedef struct {
   int64_t pool_bytes;          /* page pool size; 0 = auto */
   int32_t blocks;              /* 0 = auto: SM count x resident blocks per SM (persistent) */
   int32_t warps_per_block;     /* 0 = auto (4) */
-  int32_t shard_rank;          /* this GPU's share of the initial edge tasks: directed edge e is */
-  int32_t shard_world;         /*   processed iff e mod shard_world == shard_rank */
+  int32_t shard_rank;          /* this GPU's share of the initial edge tasks (see shard_policy); */
+  int32_t shard_world;         /*   1 = every directed edge */
   uint32_t flags;              /* TDFS_RUN_* */
+  int32_t shard_policy;        /* TDFS_SHARD_ROUND_ROBIN (default) or TDFS_SHARD_DEGREE_BALANCED */
+  int32_t reserved_;           /* 0 */
+  uint64_t* shared_cursor;     /* NULL, or a device pointer (this device's memory or a peer's, e.g. from
+                                  tdfs_shared_cursor_open) to a uint64 chunk cursor over ALL nnz directed edges,
+                                  zeroed before the job and shared by every rank's concurrent job on the same
+                                  graph (cross-GPU dynamic balancing; PAPER.md:122
+                                  omits migration).  Overrides shard_rank/world/policy: each rank takes chunks
+                                  from the shared cursor with system-scope atomics until it is exhausted. */
 } tdfs_run_opts;
 
 void tdfs_run_opts_default(tdfs_run_opts* o);
@@ -207,6 +225,24 @@ int tdfs_enumerate(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts*
 
 /* Status of the last job run in `workspace` (device-side error word), synchronising `stream`. */
 int tdfs_workspace_status(const void* workspace, void* stream);
+
+/* ------------------------------------------------------------------ multi-GPU helpers
+ * Owner rank of every directed edge under a shard policy (host only, no GPU needed):
+ *  offs[n+1], adj[nnz] a CSR as in tdfs_csr (host); owner[nnz] receives the rank in [0, world) of the
+ *  initial edge task e (the kernel's shard rank r processes exactly the edges with owner[e] == r).
+ * Errors: INVALID_ARG (world < 1, unknown policy, NULL, nnz >= 2^31 for DEGREE_BALANCED). */
+int tdfs_partition_edges(int64_t n, int64_t nnz, const int64_t* offs, const int32_t* adj, int32_t world,
+                         int32_t policy, int32_t* owner);
+
+/* A uint64 chunk cursor in this process's device memory that other processes (ranks on peer GPUs
+ * of the same node, or on the same GPU) can map: *d_cursor is the local device pointer, ipc_handle
+ * (64 bytes, cudaIpcMemHandle_t) is what the other ranks pass to tdfs_shared_cursor_open.  The
+ * cursor is zeroed on `stream` by tdfs_shared_cursor_reset before each job. */
+int tdfs_shared_cursor_create(int device, uint64_t** d_cursor, void* ipc_handle /* 64 bytes */);
+int tdfs_shared_cursor_open(int device, const void* ipc_handle, uint64_t** d_cursor);
+int tdfs_shared_cursor_reset(uint64_t* d_cursor, void* stream);
+/* Close a cursor obtained from _open (opened = 1) or free one from _create (opened = 0). */
+int tdfs_shared_cursor_close(uint64_t* d_cursor, int opened);
 
 #ifdef __cplusplus
 }

@@ -28,7 +28,8 @@
  *    placed as in DESIGN.md reading R8 (positions 0 and 1 always, later
  *    positions only when deg_Q(u) > |B^pi(u)|);
  *  - per-position node counts and the algorithmic byte count W of
- *    SURVEY.md 8(d) (sum over internal prefixes of 4*|operand| + 16 bytes);
+ *    SURVEY.md 8(d) (sum over internal prefixes of 4*|operand| + 16 bytes), and the
+ *    roofline bytes of DESIGN.md R32 (smallest Eq. (1) source per extension);
  *  - a restriction of the root edge (f(pi_0), f(pi_1)) to those whose rank in
  *    the lexicographic order of directed edges is = r (mod W_shard), used for
  *    sampled parity and the shard-sum invariant.
@@ -79,13 +80,16 @@ struct Acc {
   uint64_t count = 0;
   uint64_t nodes[9] = {0};
   uint64_t wbytes = 0;
-  uint64_t sbytes = 0;   /* R29b */
+  uint64_t sbytes = 0;   /* R32 roofline bytes */
   std::vector<int32_t> tuples;  // local tuples (enumerate)
+  std::vector<const std::vector<int32_t>*> raw;  // per position: Eq. (1) result before the checks
 };
 
 int64_t degree(const DataGraph& g, int32_t v) { return (int64_t)g.adj[v].size(); }
 
 int query_degree(const QueryGraph& q, int u) { return (int)q.nbr[u].size(); }
+
+int degree_threshold(const Job& J, int i);
 
 /* Degree filter placement, reading R8. */
 bool degree_ok(const Job& J, int i, int32_t v) {
@@ -143,16 +147,50 @@ bool in_shard(const Job& J, int32_t v0, int32_t v1) {
   return rank % J.shard_world == J.shard_rank;
 }
 
+/* Is the degree filter applied at position i (R8), and with which threshold (0 = none)? */
+int degree_threshold(const Job& J, int i) {
+  if (!J.deg_filter) return 0;
+  int dq = query_degree(*J.q, J.order[i]);
+  return (i <= 1 || dq > (int)J.bwd[i].size()) ? dq : 0;
+}
+
+/* R32: may the candidate set C(r) of an earlier position r -- the ids that passed
+ * every check at r -- serve as an Eq. (1) source for position i ("if
+ * B(u_j) is a subset of B(u_i) ... C(u_i) can be computed from C(u_j)")?  Only if every check
+ * made at r also holds for each candidate of i, so that C(r) contains C(i):
+ *   adjacency: B(r) is a subset of B(i);
+ *   label:     r has no label test, or i tests the same label;
+ *   degree:    r's threshold is at most i's own, or at most |B(i)| (a candidate of i is adjacent
+ *              to |B(i)| distinct matched vertices);
+ *   constraints: every window bound (j, sign) checked at r is also checked at i;
+ *   injectivity: checked at i against every earlier position anyway. */
+bool source_ok(const Job& J, int r, int i) {
+  for (int pj : J.bwd[r])
+    if (std::find(J.bwd[i].begin(), J.bwd[i].end(), pj) == J.bwd[i].end()) return false;
+  const int lr = J.q->label[J.order[r]], li = J.q->label[J.order[i]];
+  if (lr >= 0 && lr != li) return false;
+  const int dr = degree_threshold(J, r), di = degree_threshold(J, i);
+  if (dr > std::max(di, (int)J.bwd[i].size())) return false;
+  for (auto& c : J.cons_at[r])
+    if (std::find(J.cons_at[i].begin(), J.cons_at[i].end(), c) == J.cons_at[i].end()) return false;
+  return true;
+}
+
 /* Algorithm 1, procedure enumerate(S, i, pi, G_Q, G). */
 void enumerate(const Job& J, std::vector<int32_t>& S, int i, Acc& acc,
                std::vector<std::vector<int32_t>>& cbuf) {
   const int k = J.q->k;
   const std::vector<int32_t>& C = *candidates(J, S, i, cbuf[i]);  /* line 3 */
+  acc.raw[i] = &C;
   if (i >= 2) {                                        /* W of SURVEY 8(d) */
     for (int pj : J.bwd[i]) acc.wbytes += 4ull * (uint64_t)degree(*J.g, S[pj]) + 16ull;
-    /* R29b: 16 B per operand + 4 B x the smallest operand restricted to the ids the
-     * constraints already allow (lo <= w < hi); nothing for a count-only last position
-     * with a single operand and no label test */
+    /* R32 roofline bytes: 16 B per backward operand + 4 B x the smallest SOURCE of Eq. (1)
+     * restricted to the ids the constraints already allow (lo <= w < hi).  Sources: every
+     * backward operand N(S[j]), and the candidate set C(r) of every stored earlier position
+     * r (2 <= r <= k-2) allowed by source_ok (set-intersection reuse).
+     * No id bytes for a count-only last position: one source that alone is C(i) up to the
+     * matched vertices (a single operand, or a C(r) with B(r) = B(i)) and no label or degree
+     * test left at i. */
     int64_t lo = 0, hi = (int64_t)INT32_MAX + 1;
     for (auto& c : J.cons_at[i]) {
       if (c.second > 0) lo = std::max<int64_t>(lo, (int64_t)S[c.first] + 1);
@@ -165,7 +203,21 @@ void enumerate(const Job& J, std::vector<int32_t>& S, int i, Acc& acc,
       if (lo < hi) len = (uint64_t)(std::lower_bound(L.begin(), L.end(), hi) - std::lower_bound(L.begin(), L.end(), lo));
       mn = std::min(mn, len);
     }
-    bool count_only = (i + 1 == J.q->k) && J.bwd[i].size() == 1 && J.q->label[J.order[i]] < 0;
+    const int li = J.q->label[J.order[i]];
+    const bool no_test = li < 0 && degree_threshold(J, i) == 0;
+    bool count_only = (i + 1 == k) && J.bwd[i].size() == 1 && no_test;
+    for (int r = 2; r < i && r <= k - 2; r++) {
+      if (!source_ok(J, r, i)) continue;
+      uint64_t len = 0;  /* |C(r) within [lo, hi)|: ids of the raw list that passed r's checks */
+      for (int32_t v : *acc.raw[r])
+        if (v >= lo && v < hi && admissible(J, S, r, v)) len++;
+      mn = std::min(mn, len);
+      const bool same_b = J.bwd[r].size() == J.bwd[i].size();
+      const int lr = J.q->label[J.order[r]];
+      const bool label_done = li < 0 || lr == li;
+      const int di = degree_threshold(J, i);
+      if (i + 1 == k && same_b && label_done && (di == 0 || degree_threshold(J, r) >= di)) count_only = true;
+    }
     acc.sbytes += 16ull * J.bwd[i].size() + ((count_only || lo >= hi || mn == UINT64_MAX) ? 0ull : 4ull * mn);
   }
   for (size_t t = 0; t < C.size(); t++) {              /* line 4 */
@@ -320,6 +372,7 @@ static int match_on(const DataGraph& g,
   std::atomic<int64_t> next(lo);
   auto worker = [&](int t) {
     Acc& acc = accs[t];
+    acc.raw.assign(k, nullptr);
     std::vector<int32_t> S(k, -1);
     std::vector<std::vector<int32_t>> cbuf(k);
     std::vector<int32_t> C0;

@@ -18,7 +18,7 @@ from typing import Optional, Sequence, Tuple, Union
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.environ.get("TDFS_LIB") or os.path.join(_PKG, "libtdfs.so")  # TDFS_LIB: experiment variants
+LIB_PATH = os.path.join(_PKG, "libtdfs.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libtdfs.so not found at {LIB_PATH}: build it first "
@@ -45,8 +45,10 @@ TDFS_RUN_NO_REUSE = 4
 TDFS_RUN_NO_SHORTCUT = 8
 TDFS_RUN_NO_HUB_BITMAP = 16
 TDFS_RUN_NO_LEAF_STAGE = 32
-TDFS_RUN_NO_HASH = 64
 TDFS_RUN_ARRAY_STACKS = 128
+TDFS_RUN_NO_RANGE_TASKS = 256
+TDFS_SHARD_ROUND_ROBIN = 0
+TDFS_SHARD_DEGREE_BALANCED = 1
 TDFS_COUNT_INVALID = (1 << 64) - 1
 
 
@@ -60,7 +62,8 @@ class TdfsError(RuntimeError):
 # ----------------------------------------------------------------- structs
 class tdfs_csr(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("offs", ctypes.c_void_p), ("adj", ctypes.c_void_p),
-                ("label", ctypes.c_void_p), ("mem", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+                ("label", ctypes.c_void_p), ("mem", ctypes.c_int32), ("flags", ctypes.c_uint32),
+                ("hub_bitmap_bytes", ctypes.c_int64)]
 
 
 class tdfs_plan_opts(ctypes.Structure):
@@ -72,7 +75,8 @@ class tdfs_run_opts(ctypes.Structure):
     _fields_ = [("tau_ns", ctypes.c_int64), ("chunk", ctypes.c_int32), ("queue_ints", ctypes.c_int64),
                 ("page_bytes", ctypes.c_int32), ("page_table_entries", ctypes.c_int32),
                 ("pool_bytes", ctypes.c_int64), ("blocks", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
-                ("shard_rank", ctypes.c_int32), ("shard_world", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+                ("shard_rank", ctypes.c_int32), ("shard_world", ctypes.c_int32), ("flags", ctypes.c_uint32),
+                ("shard_policy", ctypes.c_int32), ("reserved_", ctypes.c_int32), ("shared_cursor", ctypes.c_void_p)]
 
 
 class tdfs_stats(ctypes.Structure):
@@ -101,8 +105,8 @@ SIGNATURES = {
     "tdfs_last_error": (ctypes.c_char_p, []),
     "tdfs_abi_version": (ctypes.c_int, []),
     "tdfs_load_graph": (ctypes.c_int, [ctypes.POINTER(tdfs_csr), ctypes.c_int, _vp, ctypes.POINTER(_vp)]),
-    "tdfs_load_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, ctypes.c_int, _vp,
-                                       ctypes.POINTER(_vp)]),
+    "tdfs_load_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, ctypes.c_int64, ctypes.c_int,
+                                       _vp, ctypes.POINTER(_vp)]),
     "tdfs_graph_info": (ctypes.c_int, [_vp, _i64p, _i64p, _i64p, _i32p]),
     "tdfs_graph_device_arrays": (ctypes.c_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
     "tdfs_free_graph": (None, [_vp]),
@@ -120,6 +124,12 @@ SIGNATURES = {
     "tdfs_enumerate": (ctypes.c_int, [_vp, _vp, ctypes.POINTER(tdfs_run_opts), _vp, ctypes.c_size_t, _vp, _vp,
                                       ctypes.c_uint64, _u64p, ctypes.POINTER(tdfs_stats)]),
     "tdfs_workspace_status": (ctypes.c_int, [_vp, _vp]),
+    "tdfs_partition_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, ctypes.c_int32, ctypes.c_int32,
+                                            _vp]),
+    "tdfs_shared_cursor_create": (ctypes.c_int, [ctypes.c_int, ctypes.POINTER(_vp), _vp]),
+    "tdfs_shared_cursor_open": (ctypes.c_int, [ctypes.c_int, _vp, ctypes.POINTER(_vp)]),
+    "tdfs_shared_cursor_reset": (ctypes.c_int, [_vp, _vp]),
+    "tdfs_shared_cursor_close": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tdfs_test_queue": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_uint64,
                                        ctypes.c_int64, _i32p, _i32p, _i64p, _i64p]),
     "tdfs_test_paged_write": (ctypes.c_int, [ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_uint32, _i32p,
@@ -229,7 +239,7 @@ class PlanHandle:
 
 # ----------------------------------------------------------------- graph loading
 def tdfs_load_graph(offs, adj, label=None, device: int = 0, stream=None, validate: bool = False,
-                    normalize: bool = False) -> GraphHandle:
+                    normalize: bool = False, hub_bitmap_bytes: int = 0) -> GraphHandle:
     """Load a CSR.  numpy arrays -> HOST_COPY; torch CUDA tensors -> DEVICE_BORROW (kept alive by the handle)."""
     flags = (TDFS_GRAPH_VALIDATE if validate else 0) | (TDFS_GRAPH_NORMALIZE if normalize else 0)
     keep = None
@@ -240,7 +250,7 @@ def tdfs_load_graph(offs, adj, label=None, device: int = 0, stream=None, validat
         offs, adj = offs.contiguous(), adj.contiguous()
         label = None if label is None else label.contiguous()
         c = tdfs_csr(offs.numel() - 1, adj.numel(), offs.data_ptr(), adj.data_ptr(),
-                     None if label is None else label.data_ptr(), TDFS_MEM_DEVICE_BORROW, flags)
+                     None if label is None else label.data_ptr(), TDFS_MEM_DEVICE_BORROW, flags, hub_bitmap_bytes)
         keep = (offs, adj, label)
         device = offs.device.index or 0
     else:
@@ -248,13 +258,13 @@ def tdfs_load_graph(offs, adj, label=None, device: int = 0, stream=None, validat
         adj = np.ascontiguousarray(adj, dtype=np.int32)
         label = None if label is None else np.ascontiguousarray(label, dtype=np.uint8)
         c = tdfs_csr(offs.shape[0] - 1, adj.shape[0], offs.ctypes.data, adj.ctypes.data,
-                     None if label is None else label.ctypes.data, TDFS_MEM_HOST_COPY, flags)
+                     None if label is None else label.ctypes.data, TDFS_MEM_HOST_COPY, flags, hub_bitmap_bytes)
     out = _vp()
     _check(_lib.tdfs_load_graph(ctypes.byref(c), device, _stream_ptr(stream, device), ctypes.byref(out)))
     return GraphHandle(out.value, device, keep)
 
 
-def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None) -> GraphHandle:
+def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None, hub_bitmap_bytes: int = 0) -> GraphHandle:
     """Load an undirected edge list ((m, 2) int array, host) -- normalised by the library."""
     e = np.ascontiguousarray(np.asarray(edges, dtype=np.int32).reshape(-1, 2))
     src = np.ascontiguousarray(e[:, 0])
@@ -262,8 +272,8 @@ def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None) -> 
     lab = None if label is None else np.ascontiguousarray(label, dtype=np.uint8)
     out = _vp()
     _check(_lib.tdfs_load_edges(int(n), e.shape[0], src.ctypes.data, dst.ctypes.data,
-                                None if lab is None else lab.ctypes.data, device, _stream_ptr(stream, device),
-                                ctypes.byref(out)))
+                                None if lab is None else lab.ctypes.data, int(hub_bitmap_bytes), device,
+                                _stream_ptr(stream, device), ctypes.byref(out)))
     return GraphHandle(out.value, device)
 
 
@@ -412,7 +422,8 @@ def tdfs_enumerate_chunks(g: GraphHandle, p: PlanHandle, chunk_cap: int, opts: O
         return
     out = torch.empty(chunk_cap * k, dtype=torch.int32, device=f"cuda:{g.device}")
     host = torch.empty(chunk_cap * k, dtype=torch.int32, pin_memory=True)
-    S = max(1, -(-2 * total // chunk_cap))  # ~2x headroom for uneven sub-shards
+    # ~2x headroom for uneven sub-shards, capped (a sub-shard that overflows is split again)
+    S = min(max(1, -(-2 * total // chunk_cap)), 4096)
     todo = [(base_r + base_w * s, base_w * S) for s in range(S - 1, -1, -1)]
     done = 0
     while todo:
@@ -442,6 +453,51 @@ def tdfs_enumerate_chunks(g: GraphHandle, p: PlanHandle, chunk_cap: int, opts: O
 
 def tdfs_workspace_status(workspace, stream=None, device: int = 0) -> int:
     return _check(_lib.tdfs_workspace_status(workspace.data_ptr(), _stream_ptr(stream, device)))
+
+
+# ----------------------------------------------------------------- multi-GPU helpers
+def tdfs_partition_edges(offs, adj, world: int, policy: int = TDFS_SHARD_ROUND_ROBIN) -> np.ndarray:
+    """Owner rank of every directed edge (host CSR numpy arrays) under a shard policy (tdfs.h)."""
+    offs = np.ascontiguousarray(offs, dtype=np.int64)
+    adj = np.ascontiguousarray(adj, dtype=np.int32)
+    owner = np.empty(max(1, adj.shape[0]), dtype=np.int32)
+    _check(_lib.tdfs_partition_edges(offs.shape[0] - 1, adj.shape[0], offs.ctypes.data, adj.ctypes.data,
+                                     int(world), int(policy), owner.ctypes.data))
+    return owner[: adj.shape[0]]
+
+
+class SharedCursor:
+    """A uint64 chunk cursor in one rank's device memory, mapped by the others through CUDA IPC
+    (tdfs_shared_cursor_*; cross-GPU dynamic balancing)."""
+
+    def __init__(self, device: int, handle: Optional[bytes] = None):
+        self.device = device
+        p = _vp()
+        if handle is None:
+            buf = ctypes.create_string_buffer(64)
+            _check(_lib.tdfs_shared_cursor_create(device, ctypes.byref(p), buf))
+            self.handle = buf.raw
+            self.opened = 0
+        else:
+            self.handle = bytes(handle)
+            _check(_lib.tdfs_shared_cursor_open(device, ctypes.create_string_buffer(self.handle, 64),
+                                                ctypes.byref(p)))
+            self.opened = 1
+        self.ptr = p.value
+
+    def reset(self, stream=None):
+        _check(_lib.tdfs_shared_cursor_reset(self.ptr, _stream_ptr(stream, self.device)))
+
+    def close(self):
+        if self.ptr:
+            _check(_lib.tdfs_shared_cursor_close(self.ptr, self.opened))
+            self.ptr = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 # ----------------------------------------------------------------- test hooks

@@ -23,7 +23,7 @@ INCLUDE = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libtdfs.so")
 BUILD = os.path.join(PKG, "build")
 
-SOURCES = ["capi.cpp", "planner.cpp", "graph.cu", "match.cu", "test_hooks.cu"]
+SOURCES = ["capi.cpp", "planner.cpp", "graph.cu", "match.cu", "shard.cpp", "test_hooks.cu"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

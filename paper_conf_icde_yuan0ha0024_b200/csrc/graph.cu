@@ -112,6 +112,23 @@ int validate_host(int64_t n, int64_t nnz, const int64_t* offs, const int32_t* ad
   return TDFS_OK;
 }
 
+// Cheap host check without VALIDATE: offsets monotone and ids in [0, n) (the kernels index with them).
+int check_host_ids(int64_t n, int64_t nnz, const int64_t* offs, const int32_t* adj) {
+  if (offs[0] != 0 || offs[n] != nnz) return fail(TDFS_E_GRAPH_FORMAT, "load: offs[0] != 0 or offs[n] != nnz");
+  std::atomic<int> bad(0);
+  parallel_for(n, [&](int64_t lo, int64_t hi) {
+    for (int64_t v = lo; v < hi; v++)
+      if (offs[v + 1] < offs[v]) { bad = 1; return; }
+  });
+  if (bad.load()) return fail(TDFS_E_GRAPH_FORMAT, "load: offsets decrease");
+  parallel_for(nnz, [&](int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; i++)
+      if (adj[i] < 0 || adj[i] >= n) { bad = 2; return; }
+  });
+  if (bad.load()) return fail(TDFS_E_ID_RANGE, "load: neighbour id outside [0, n)");
+  return TDFS_OK;
+}
+
 // ------------------------------------------------------------- device helpers
 __global__ void fill_src_kernel(const int64_t* __restrict__ offs, int64_t n, int32_t* __restrict__ src) {
   const int lane = threadIdx.x & 31;
@@ -138,10 +155,11 @@ __global__ void scan_graph_kernel(const int64_t* __restrict__ offs, const int32_
       else dmax = max(dmax, (unsigned long long)(e - b));
       if (label) lmax = max(lmax, (unsigned long long)label[v]);
     }
-    if (!validate || e < b) continue;
+    if (e < b) continue;
     for (int64_t i = b + lane; i < e; i += 32) {
       int32_t w = adj[i];
-      if (w < 0 || w >= n) { flags |= 2; continue; }
+      if (w < 0 || w >= n) { flags |= 2; continue; }  // always: an id >= n would be read out of bounds
+      if (!validate) continue;
       if (w == v || (i > b && adj[i - 1] >= w)) flags |= 1;
       // symmetry: v must be in N(w)
       int64_t lo = offs[w], hi = offs[w + 1];
@@ -173,17 +191,16 @@ __global__ void hub_bits_kernel(const int64_t* __restrict__ offs, const int32_t*
 // Hub adjacency bitmaps: the highest-degree vertices (degree >= 256,
 // at most `budget` bytes of bitmaps) get an n-bit membership bitmap so that probing
 // w in N(hub) during Eq. (1) is one load instead of a binary search over a long list.
-int build_hub_bitmaps(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs, std::vector<int32_t>& hub_vertices) {
+int build_hub_bitmaps(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs, int64_t budget) {
   const long long words = (G.n + 31) / 32;
-  if (G.n == 0 || words == 0) return TDFS_OK;
-  long long budget = 256ll << 20;  // measured on config 2: 16/64/256/1024 MB -> c4 2029/1416/1350/1350 ms
-  if (const char* e = getenv("TDFS_HUB_BUDGET_MB")) budget = atoll(e) << 20;
+  if (G.n == 0 || words == 0 || budget < 0) return TDFS_OK;
+  // default 256 MB -- measured on config 2: 16/64/256/1024 MB -> c4 2029/1416/1350/1350 ms
+  if (budget == 0) budget = kHubBudgetDefault;
   const long long max_hubs = budget / (words * 4);
   if (max_hubs <= 0) return TDFS_OK;
   cudaError_t e;
   std::vector<std::pair<int64_t, int32_t>> cand;
-  int64_t min_deg = 256;
-  if (const char* e = getenv("TDFS_HUB_MIN_DEG")) min_deg = std::max(1ll, atoll(e));  // tuning knob (experiments)
+  const int64_t min_deg = kHubMinDeg;
   for (int64_t v = 0; v < G.n; v++) {
     int64_t d = offs[v + 1] - offs[v];
     if (d >= min_deg) cand.push_back({-d, (int32_t)v});
@@ -217,81 +234,18 @@ int build_hub_bitmaps(Graph& G, cudaStream_t st, const std::vector<int64_t>& off
   e = cudaStreamSynchronize(st);
   cudaFree(d_vert);
   if (e != cudaSuccess) return cuda_fail(e, "hubs: build");
-  hub_vertices = hub_vertex;
   return TDFS_OK;
 }
 
-// Per-vertex open-addressing hash sets of the adjacency lists:
-// vertex v with deg(v) >= kHashMinDeg owns T_v = next_pow2(2 deg(v)) int32 slots
-// (load factor <= 1/2) at hoff[v]; w sits at or after slot fib(w) >> (32 - log2 T_v),
-// linear probing, EMPTY = -1.  Membership w in N(v) during Eq. (1) then costs one
-// aligned 16-byte group load (rarely two) instead of log2 deg(v) dependent loads.
-// The sorted CSR stays the primary copy (streamed operands, windows, merge).
-__global__ void hash_fill_kernel(const int64_t* __restrict__ offs, const int32_t* __restrict__ adj, int64_t n,
-                                 const int64_t* __restrict__ hoff, int32_t* __restrict__ slots) {
-  const int64_t nwarps = (int64_t)gridDim.x * blockDim.x / 32;
-  const int lane = threadIdx.x & 31;
-  for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; v < n; v += nwarps) {
-    const int64_t h0 = hoff[v], T = hoff[v + 1] - h0;
-    if (T == 0) continue;
-    const int sh = 32 - (31 - __clz((int)T));  // 32 - log2 T
-    for (int64_t e = offs[v] + lane; e < offs[v + 1]; e += 32) {
-      const int32_t w = adj[e];
-      uint32_t s = ((uint32_t)w * 2654435769u) >> sh;
-      for (;;) {
-        const int old = atomicCAS(slots + h0 + s, -1, w);
-        if (old == -1 || old == w) break;
-        s = (s + 1) & (uint32_t)(T - 1);
-      }
-    }
-  }
-}
-
-int build_hash_index(Graph& G, cudaStream_t st, const std::vector<int64_t>& offs,
-                     const std::vector<int32_t>& hub_vertices) {
-  G.hash_min_deg = kHashMinDeg;
-  if (const char* e = getenv("TDFS_HASH_MIN_DEG")) G.hash_min_deg = atoll(e);  // tuning knob (experiments)
-  if (G.n == 0 || G.hash_min_deg <= 0) return TDFS_OK;
-  // hubs are probed through their bitmaps everywhere, so they get no hash set
-  std::vector<char> is_hub((size_t)G.n, 0);
-  for (int32_t v : hub_vertices) is_hub[v] = 1;
-  std::vector<int64_t> hoff((size_t)G.n + 1, 0);
-  for (int64_t v = 0; v < G.n; v++) {
-    const int64_t d = offs[v + 1] - offs[v];
-    int64_t T = 0;
-    if (d >= G.hash_min_deg && !is_hub[v]) {
-      T = 4;
-      while (T < 2 * d) T <<= 1;
-    }
-    hoff[v + 1] = hoff[v] + T;
-  }
-  if (hoff[G.n] == 0) return TDFS_OK;
-  cudaError_t e;
-  if ((e = cudaMalloc(&G.d_hoff, sizeof(int64_t) * (G.n + 1))) != cudaSuccess ||
-      (e = cudaMalloc(&G.d_hslots, sizeof(int32_t) * (size_t)hoff[G.n])) != cudaSuccess)
-    return fail(TDFS_E_OOM, "hash index: alloc");
-  G.hash_slots = hoff[G.n];
-  cudaMemcpyAsync(G.d_hoff, hoff.data(), sizeof(int64_t) * (G.n + 1), cudaMemcpyHostToDevice, st);
-  cudaMemsetAsync(G.d_hslots, 0xff, sizeof(int32_t) * (size_t)hoff[G.n], st);
-  int sms = 148;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, G.device);
-  hash_fill_kernel<<<sms * 8, 256, 0, st>>>(G.d_offs, G.d_adj, G.n, G.d_hoff, G.d_hslots);
-  if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "hash index: build");
-  return TDFS_OK;
-}
-
-int build_indexes(Graph& G, cudaStream_t st) {
+int build_indexes(Graph& G, cudaStream_t st, int64_t hub_budget) {
   std::vector<int64_t> offs((size_t)G.n + 1);
   cudaError_t e = cudaMemcpyAsync(offs.data(), G.d_offs, sizeof(int64_t) * (G.n + 1), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   if (e != cudaSuccess) return cuda_fail(e, "index: offs copy");
-  std::vector<int32_t> hubs;
-  int rc = build_hub_bitmaps(G, st, offs, hubs);
-  if (rc == TDFS_OK) rc = build_hash_index(G, st, offs, hubs);
-  return rc;
+  return build_hub_bitmaps(G, st, offs, hub_budget);
 }
 
-int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enforce = false) {
+int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enforce, int64_t hub_budget) {
   cudaError_t e;
   if ((e = cudaMalloc(&G.d_src, sizeof(int32_t) * (size_t)std::max<int64_t>(G.nnz, 1))) != cudaSuccess)
     return fail(TDFS_E_OOM, std::string("load: src array: ") + cudaGetErrorString(e));
@@ -309,13 +263,13 @@ int finish_device_graph(Graph& G, cudaStream_t st, bool scan_on_device, bool enf
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaFree(d_out);
     if (e != cudaSuccess) return cuda_fail(e, "load: scan");
-    if (enforce && (h[1] & 2)) return fail(TDFS_E_ID_RANGE, "validate (device): id out of range");
+    if (h[1] & 2) return fail(TDFS_E_ID_RANGE, "load (device scan): id out of range [0, n)");
     if (enforce && (h[1] & 1)) return fail(TDFS_E_GRAPH_FORMAT, "validate (device): bad CSR (order/dup/self-loop/asymmetric/offs)");
     G.dmax = (int64_t)h[0];
     G.nlabels = G.d_label ? (int32_t)h[2] + 1 : 1;
   }
   if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "load: sync");
-  return build_indexes(G, st);
+  return build_indexes(G, st, hub_budget);
 }
 
 void release(Graph& G) {
@@ -327,9 +281,7 @@ void release(Graph& G) {
   cudaFree(G.d_src);
   cudaFree(G.d_hub_id);
   cudaFree(G.d_hub_bits);
-  cudaFree(G.d_hoff);
-  cudaFree(G.d_hslots);
-  G.d_hoff = nullptr; G.d_hslots = nullptr; G.hash_slots = 0;
+  free_shard_lists(&G);
   G.d_offs = nullptr; G.d_adj = nullptr; G.d_label = nullptr; G.d_src = nullptr;
   G.d_hub_id = nullptr; G.d_hub_bits = nullptr; G.n_hubs = 0;
 }
@@ -402,15 +354,16 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
       G.nnz = offs[c->n];
       host_stats(G, offs.data(), c->label);
       rc = upload(G, offs.data(), adj.data(), c->label, st);
-      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false);  // sync inside: host vectors outlive copies
+      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, c->hub_bitmap_bytes);  // sync inside: host vectors outlive copies
     } else {
       if (c->flags & TDFS_GRAPH_VALIDATE) rc = validate_host(c->n, c->nnz, c->offs, c->adj);
+      else rc = check_host_ids(c->n, c->nnz, c->offs, c->adj);  // cheap: ids in [0, n), offsets sane
       G.nnz = c->nnz;
       if (rc == TDFS_OK) {
         host_stats(G, c->offs, c->label);
         rc = upload(G, c->offs, c->adj, c->label, st);
       }
-      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false);
+      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, c->hub_bitmap_bytes);
     }
   } else {
     G.owns_csr = false;
@@ -419,7 +372,7 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
     G.d_adj = const_cast<int32_t*>(c->adj);
     G.d_label = const_cast<uint8_t*>(c->label);
     // d_max and the label count come from a device scan; VALIDATE adds the format checks
-    rc = finish_device_graph(G, st, true, (c->flags & TDFS_GRAPH_VALIDATE) != 0);
+    rc = finish_device_graph(G, st, true, (c->flags & TDFS_GRAPH_VALIDATE) != 0, c->hub_bitmap_bytes);
   }
   if (rc != TDFS_OK) {
     release(G);
@@ -431,7 +384,7 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
 }
 
 extern "C" int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const int32_t* dst, const uint8_t* label,
-                               int device, void* stream, tdfs_graph** out) {
+                               int64_t hub_bitmap_bytes, int device, void* stream, tdfs_graph** out) {
   if (!out || n < 0 || m < 0 || (m > 0 && (!src || !dst))) return fail(TDFS_E_INVALID_ARG, "load_edges: bad args");
   if (n >= kMaxN) return fail(TDFS_E_ID_RANGE, "load_edges: n >= 2^31 - 2");
   std::atomic<int> bad(0);
@@ -454,7 +407,7 @@ extern "C" int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const i
   G.nnz = offs[n];
   host_stats(G, offs.data(), label);
   int rc = upload(G, offs.data(), adj.data(), label, st);
-  if (rc == TDFS_OK) rc = finish_device_graph(G, st, false);
+  if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, hub_bitmap_bytes);
   if (rc != TDFS_OK) {
     release(G);
     delete h;

@@ -28,11 +28,17 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // list and staged in shared memory; each leaf is then
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
+constexpr int kBlockThreads = 128;  // matching-kernel block size (its __launch_bounds__)
 constexpr int kLeafStage = 512;  // default shared-memory ids per warp for the leaf set F
-// Adjacency hash index: off by default (measured slower than cached binary search on the
-// L2-resident config 2); TDFS_HASH_MIN_DEG=d (e.g. 32) at load time builds it for
-// non-hub vertices of degree >= d.
-constexpr int64_t kHashMinDeg = 0;
+// Hub bitmaps (graph.cu): vertices of degree >= kHubMinDeg, highest first, within the budget
+constexpr int64_t kHubMinDeg = 256;
+constexpr int64_t kHubBudgetDefault = 256ll << 20;
+// Eq. (1) / leaf-batch cost model (measured on config 2; fixed, no run-time knobs)
+constexpr int kMergeRatio = 4;      // probe by warp merge when |B| <= 4 |A remaining|, else binary search
+constexpr int kUaHub = 4;           // stream A: per-element cost of probing a hub bitmap of N(x)
+constexpr int kUbRef = 4;           // stream B: per-element cost of probing a referenced F's bitmap
+constexpr int kRangeMin = 32;       // range tasks: >= 32 siblings each ...
+constexpr int kRangeMaxT = 32;      // ... and <= 32 tasks per split
 struct DevPlan {
   int32_t k;
   int32_t order[kMaxK];          // query vertex at position p (enumerate output mapping)
@@ -46,6 +52,10 @@ struct DevPlan {
   int32_t reuse_enabled;         // set-intersection result reuse on
   int8_t reuse[kMaxK + 1];       // stored position r whose candidate list C(r) is a superset start for p, -1 none
   uint8_t shortcut[kMaxK + 1];   // last position: count without scanning; bit0 valid with reuse, bit1 without
+  // roofline bytes (R32, STATS only): stored positions r whose C(r) may serve as an Eq. (1)
+  // source of p (every reuse candidate, not only the chosen one), and "p is count-only"
+  uint32_t src_mask[kMaxK + 1];
+  uint8_t cnt_only[kMaxK + 1];
   // leaf staging (position k-1 split into the virtual position kVF and the S[k-2] part)
   int8_t lf_on;                  // k >= 4 and B(u_{k-1}) has an operand at a position <= k-3
   int8_t lf_var;                 // N(S[k-2]) is an operand of position k-1
@@ -78,10 +88,9 @@ struct Graph {
   int32_t* d_hub_id = nullptr;     // [n], -1 for non-hubs
   uint32_t* d_hub_bits = nullptr;  // [n_hubs][hub_words]
   int64_t n_hubs = 0, hub_words = 0, hub_min_deg = 0;
-  // per-vertex adjacency hash sets (deg >= hash_min_deg), DESIGN.md "hash index"
-  int64_t* d_hoff = nullptr;       // [n+1] slot offsets, T_v = hoff[v+1]-hoff[v] (0 or a power of two)
-  int32_t* d_hslots = nullptr;     // EMPTY = -1
-  int64_t hash_slots = 0, hash_min_deg = 0;
+  // degree-balanced shard task lists, built on first use per (rank, world) (shard.cpp)
+  struct ShardList { int32_t rank, world; int32_t* d_tasks; int64_t n; };
+  mutable std::vector<ShardList> shard_lists;
 };
 
 // ---------------------------------------------------------------- device job
@@ -133,29 +142,19 @@ struct KParams {
   int32_t E;                   // page-table entries per level
   int32_t array_stacks;        // ablation: contiguous per-warp-level arrays of E pages (identity page tables)
   int64_t tau_ns;              // < 0: infinity
-  int32_t merge_ratio;         // Eq. (1) probe: merge when |B| <= merge_ratio * |A remaining|
-  int32_t merge_ratio_hash;    // the same when B has a hash set (probing it is one load per candidate)
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
   int32_t meta_off;            // shared-memory layout: byte offset of the warps' leaf-batch entries
-  int32_t range_split;
-  int32_t range_min, range_maxt;  // range tasks: >= range_min siblings each, <= range_maxt tasks per split
-  int32_t range_mode;          // 0 auto (slice unless position 2's list is reused), 1 slice, 2 whole list
-  int32_t reuse2_used;
-  int32_t range_ok;            // the plan uses range tasks (see launch_job)         // a later position / the leaf set reuses position 2's list (range tasks build it whole)         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling)
-  int32_t leaf_flat;           // staged leaves: flattened batch streams (else one leaf at a time)
-  int32_t lf_byref;            // leaf staging: reference F in place when the plan allows (else materialise)
-  int32_t lf_cost_g;
-  int32_t lf_cost_h;
-  int32_t ua_hub, ub_ref;      // flat leaf batches: per-element cost of a bitmap probe in stream A / B           // leaf staging cost model: extra cost of a hash probe over a bitmap probe           // leaf staging cost model: one dependent global load in shared-memory steps
-  int32_t coop_window;         // constraint windows by warp-cooperative 32-ary search (else per-lane binary)
-  int32_t bsearch_variant;     // 0 halving, 1 power-of-two (experiments)
+  int32_t range_split;         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling, R30)
+  int32_t range_ok;            // the plan uses range tasks (see launch_job)
+  int32_t reuse2_used;         // a later position / the leaf set reuses position 2's list (range tasks build it whole)
+  // initial edge tasks: j -> directed edge task_edges[j] (shard list) or shard_rank + j * shard_world
+  const int32_t* task_edges;   // nullptr = arithmetic shard
+  unsigned long long* gcursor; // chunk cursor: this job's counter, or a cross-rank shared one (NEXT-3)
+  int32_t gshared;             // gcursor is shared across ranks / devices: system-scope atomics
   // hub bitmaps (nullptr when off)
   const int32_t* hub_id;
   const uint32_t* hub_bits;
   long long hub_words;
-  // adjacency hash sets (nullptr when off)
-  const int64_t* hoff;
-  const int32_t* hslots;
   // enumerate
   int32_t* out;
   unsigned long long cap;
@@ -178,6 +177,11 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
                int64_t* n_trace);
 int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int* out);
 const Graph* graph_of(const tdfs_graph* g);
+// host partition of the directed edges (tdfs_partition_edges) and the device task list of one rank
+int partition_owner(int64_t n, int64_t nnz, const int64_t* offs, const int32_t* adj, int world, int policy,
+                    int32_t* owner);
+int shard_task_list(const Graph* g, int rank, int world, int policy, const int32_t** d_tasks, int64_t* n_tasks);
+void free_shard_lists(const Graph* g);
 const Plan* plan_of(const tdfs_plan* p);
 
 }  // namespace tdfs

@@ -44,13 +44,16 @@ namespace {
 #include "prims.cuh"
 
 // per-leaf entry of a flat leaf batch (shared memory, one per lane of the batch)
-struct LeafMeta {
+struct __align__(16) LeafMeta {
   long long b0;  // N(x) = adj[b0, b0 + deg)
   int deg;
   int hid;       // hub bitmap row of x, -1 = none
-  int lo, hi;    // F window of this leaf: F[lo, hi)
+  int lo, hi;    // stream B: F window of this leaf F[lo, hi); stream A: N(x)[lo, hi), the entries inside
+                 // [F_min, F_max] (the range its probes search)
+  int s, e;      // streamed element range: stream A F-coordinates [s, e) of the 16-byte aligned F,
+                 // stream B N(x) entries [b0 + s, b0 + e) (narrowed to [F_min, F_max])
 };
-// 32 entries + 33 prefix ints, padded to 16 B; with the 2 KB F stage, 16 blocks x 4 warps fit an SM
+// 32 entries + 33 prefix ints, padded to 16 B
 constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144;
 __host__ __device__ inline size_t smem_meta_offset(int wpb, int fcap) {
   return ((size_t)wpb * fcap * sizeof(int) + 15) & ~(size_t)15;
@@ -100,16 +103,6 @@ __device__ __forceinline__ long long paged_lower_bound(const KParams& P, const u
   return lo;
 }
 
-// lower_bound of v in the shared-memory list F[lo, hi) (all lanes, same v: broadcast reads)
-__device__ __forceinline__ int smem_lower_bound(const int* F, int lo, int hi, int v) {
-  while (lo < hi) {
-    const int mid = (lo + hi) >> 1;
-    if (F[mid] < v) lo = mid + 1;
-    else hi = mid;
-  }
-  return lo;
-}
-
 // Warp-cooperative lower_bound of v in the sorted global list L[0, n): each round the 32
 // lanes sample the remaining range at 32 evenly spaced points (one load per lane) and keep
 // one stride, so a list of n ids takes ceil(log32 n) dependent loads instead of log2 n.
@@ -144,6 +137,46 @@ __device__ __forceinline__ long long warp_paged_lower_bound(const KParams& P, co
   return lo + __popc(__ballot_sync(FULL, less));
 }
 
+// STATS only (roofline bytes R32): |C(r) within [lo, hi)| from the definition, for a stored
+// position r whose list this warp did not build (a <v1,v2,v3> or range task): the ids of the
+// intersection of r's backward lists inside r's window and [lo, hi) that pass r's injectivity,
+// label and degree tests.  Streams r's first operand, binary-searches the others.
+template <bool STATS>
+__device__ long long source_size_def(const KParams& P, Ctx<STATS>& c, int r, int lo, int hi) {
+  const DevPlan& pl = P.plan;
+  const int lane = c.lane;
+  lo = max(lo, (int)__reduce_max_sync(FULL, ((pl.lo_mask[r] >> lane) & 1u) ? (unsigned)(c.sreg + 1) : 0u));
+  hi = min(hi, (int)__reduce_min_sync(FULL, ((pl.hi_mask[r] >> lane) & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX));
+  if (lo >= hi) return 0;
+  const uint32_t bm = pl.bwd[r];
+  const int x0 = getS(c.sreg, __ffs(bm) - 1);
+  const long long b0 = __ldg(P.offs + x0), e0 = __ldg(P.offs + x0 + 1);
+  const long long s = b0 + warp_lower_bound(P.adj + b0, e0 - b0, lo, lane);
+  long long total = 0;
+  for (long long base = s; base < e0; base += 32) {
+    const long long i = base + lane;
+    const int v = i < e0 ? __ldg(P.adj + i) : INT_MAX;
+    bool ok = i < e0 && v < hi;
+    for (uint32_t m = bm & (bm - 1); m; m &= m - 1) {
+      const int x = getS(c.sreg, __ffs(m) - 1);
+      if (ok) {
+        const long long b = __ldg(P.offs + x), e = __ldg(P.offs + x + 1);
+        const int pos = lower_bound_dev(P.adj + b, (int)(e - b), v);
+        ok = pos < e - b && __ldg(P.adj + b + pos) == v;
+      }
+    }
+    for (uint32_t m = pl.inj_mask[r]; m; m &= m - 1) {
+      const int sj = getS(c.sreg, __ffs(m) - 1);
+      ok = ok && v != sj;
+    }
+    if (ok && pl.label[r] >= 0) ok = (P.label ? (int)__ldg(P.label + v) : 0) == pl.label[r];
+    if (ok && pl.deg_min[r] > 0) ok = (__ldg(P.offs + v + 1) - __ldg(P.offs + v)) >= pl.deg_min[r];
+    total += __popc(__ballot_sync(FULL, ok));
+    if (!__any_sync(FULL, i < e0 && v < hi)) break;
+  }
+  return total;
+}
+
 // Candidate generation for position d (Eq. 1 + fused filters).
 // MODE_OUT: 0 = store into the paged level of d; 1 = count only (last position);
 //           2 = enumerate (last position); 3 = stage into shared memory (d = kVF, the
@@ -172,16 +205,10 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   const int sj = __shfl_sync(FULL, c.sreg, jt);
   long long ob = 0, oe = 0;
   int hid = -1;
-  long long hb = 0;  // hash set of the operand: slots [hb, hb + hT), hT = 0 if none
-  unsigned hT = 0;
   if (lane < nops) {
     ob = __ldg(P.offs + sj);
     oe = __ldg(P.offs + sj + 1);
     if (P.hub_id) hid = __ldg(P.hub_id + sj);
-    if (P.hoff) {
-      hb = __ldg(P.hoff + sj);
-      hT = (unsigned)(__ldg(P.hoff + sj + 1) - hb);
-    }
   }
   // a range task re-extends part of a level-2 list its splitter already counted (STATS only)
   const bool counted = STATS && MODE_OUT != 3 && !(d == 2 && c.w2mode != 0);
@@ -200,7 +227,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     lo = max(lo, c.w2lo);
     hi = min(hi, c.w2hi);
   }
-  if (counted) {  // roofline bytes R29b: 16 B per operand + 4 B x smallest windowed operand
+  if (counted) {  // roofline bytes R32: 16 B per operand + 4 B x the smallest windowed Eq. (1) source
     const bool mine = (bm_all >> lane) & 1u;
     unsigned wlen = UINT_MAX;
     if (mine && lo < hi) {
@@ -210,14 +237,27 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       const int z = hi < INT_MAX ? a + lower_bound_dev(P.adj + b + a, n - a, hi) : n;
       wlen = (unsigned)(z - a);
     }
-    const unsigned mn = __reduce_min_sync(FULL, wlen);
+    unsigned mn = __reduce_min_sync(FULL, wlen);
+    if (lo < hi)
+      for (uint32_t sm = pl.src_mask[d]; sm; sm &= sm - 1) {  // stored candidate sets C(r) (reuse sources)
+        const int rr = __ffs(sm) - 1;
+        long long len;
+        if (rr == 2 && !allow_reuse2) {
+          len = source_size_def(P, c, rr, lo, hi);  // level 2 not built by this warp: from the definition
+        } else {
+          const uint32_t* tb = c.tables + (size_t)(rr - 2) * P.E;
+          const long long rs = __shfl_sync(FULL, c.lsize, rr);
+          const long long a = lo > 0 ? warp_paged_lower_bound(P, tb, 0, rs, lo, lane) : 0;
+          len = (hi < INT_MAX ? warp_paged_lower_bound(P, tb, a, rs, hi, lane) : rs) - a;
+        }
+        mn = min(mn, (unsigned)len);
+      }
     const int nall = __popc(bm_all);
-    const bool count_only = (d == pl.k - 1) && nall == 1 && pl.label[d] < 0 && pl.deg_min[d] == 0;
-    if (lane == 0) c.sbytes += 16ull * nall + ((lo >= hi || count_only || mn == UINT_MAX) ? 0ull : 4ull * mn);
+    if (lane == 0) c.sbytes += 16ull * nall + ((lo >= hi || pl.cnt_only[d] || mn == UINT_MAX) ? 0ull : 4ull * mn);
   }
   if (lo >= hi) return 0;
   const bool windowed = (lo > 0 || hi < INT_MAX);
-  if (windowed && P.coop_window) {
+  if (windowed) {
     // warp-cooperative window search, one operand at a time (ceil(log32 n) dependent loads)
     for (int t = 0; t < nops; t++) {
       const long long tb = __shfl_sync(FULL, ob, t), te = __shfl_sync(FULL, oe, t);
@@ -225,13 +265,6 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       const long long b = hi < INT_MAX ? a + warp_lower_bound(P.adj + tb + a, te - tb - a, hi, lane) : te - tb;
       if (lane == t) { ob = tb + a; oe = tb + b; }
     }
-  } else if (lane < nops && windowed) {
-    const int32_t* L = P.adj + ob;
-    const int n = (int)(oe - ob);
-    const int a = lo > 0 ? lower_bound_dev(L, n, lo) : 0;
-    const int b = hi < INT_MAX ? a + lower_bound_dev(L + a, n - a, hi) : n;
-    oe = ob + b;
-    ob = ob + a;
   }
   // the reused list, windowed
   const uint32_t* rtable = nullptr;
@@ -248,10 +281,8 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       ra_known = (lo == getS(c.sreg, r) + 1);
     }
     if (ra_known) ra = r0;
-    else if (P.coop_window) ra = lo > 0 ? warp_paged_lower_bound(P, rtable, r0, rsize, lo, lane) : 0;
-    else ra = lo > 0 ? paged_lower_bound(P, rtable, r0, rsize, lo) : 0;
-    if (P.coop_window) rb = hi < INT_MAX ? warp_paged_lower_bound(P, rtable, ra, rsize, hi, lane) : rsize;
-    else rb = hi < INT_MAX ? paged_lower_bound(P, rtable, ra, rsize, hi) : rsize;
+    else ra = lo > 0 ? warp_paged_lower_bound(P, rtable, r0, rsize, lo, lane) : 0;
+    rb = hi < INT_MAX ? warp_paged_lower_bound(P, rtable, ra, rsize, hi, lane) : rsize;
     if (ra >= rb) return 0;
   }
   const uint32_t injm = pl.inj_mask[d];
@@ -328,7 +359,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       if (th >= 0) {
         // hub operand: one bitmap load per candidate (v is inside the window already)
         if (ok) ok = (__ldg(P.hub_bits + (long long)th * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
-      } else if ((te - tb) <= (long long)(__shfl_sync(FULL, hT, t) ? P.merge_ratio_hash : P.merge_ratio) * (eA - base)) {
+      } else if ((te - tb) <= (long long)kMergeRatio * (eA - base)) {
         // warp merge: walk B in coalesced 32-id chunks until a chunk reaches the batch max
         const int amax = __shfl_sync(FULL, v, last_lane);
         bool found = false;
@@ -347,15 +378,10 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
         }
         ok = ok && found;
         if (lane == t) ob = min(ptr, te);
-      } else if (const unsigned tT = __shfl_sync(FULL, hT, t)) {
-        // hashed operand: one aligned 16-byte group load per candidate (rarely two)
-        const long long th0 = __shfl_sync(FULL, hb, t);
-        if (ok) ok = hash_contains(P.hslots, th0, tT, v);
       } else {
         int pos = (int)(te - tb);
         const bool probe = inr && (ok || lane == last_lane);
-        if (probe) pos = P.bsearch_variant ? lower_bound_pow2(P.adj + tb, (int)(te - tb), v)
-                                           : lower_bound_dev(P.adj + tb, (int)(te - tb), v);
+        if (probe) pos = lower_bound_dev(P.adj + tb, (int)(te - tb), v);
         if (ok) ok = (pos < te - tb) && __ldg(P.adj + tb + pos) == v;
         const int adv = __shfl_sync(FULL, pos, last_lane);
         if (lane == t) ob = tb + adv;
@@ -399,17 +425,9 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   return total;
 }
 
-// Leaf of a count job with the staged set F = sF[0, nF) (sorted, all S[k-2]-independent
-// filters applied): |F ∩ window(x) ∩ N(x)| when N(x) is an operand, else |F ∩ window(x)|
-// minus x itself, where x = S[k-2].  Either F is streamed
-// from shared memory and N(x) probed (hub bitmap, else per-lane binary search with an
-// advancing lower bound), or N(x) is streamed with coalesced loads -- first narrowed to
-// [F_min, F_max] by a warp-cooperative search -- and F probed in shared memory.
-// Per-vertex probe metadata of N(x): CSR range, hub bitmap row, hash set.
+// Per-vertex probe metadata of N(x): CSR range, hub bitmap row.
 struct VMeta {
   long long b0, b1;  // N(x) = adj[b0, b1)
-  long long hb;      // hash slots [hb, hb + hT)
-  unsigned hT;       // 0 = no hash set
   int hid;           // hub bitmap row, -1 = none
 };
 
@@ -418,35 +436,17 @@ __device__ __forceinline__ VMeta load_vmeta(const KParams& P, int x) {
   m.b0 = __ldg(P.offs + x);
   m.b1 = __ldg(P.offs + x + 1);
   m.hid = P.hub_id ? __ldg(P.hub_id + x) : -1;
-  m.hb = 0;
-  m.hT = 0;
-  if (P.hoff) {
-    m.hb = __ldg(P.hoff + x);
-    m.hT = (unsigned)(__ldg(P.hoff + x + 1) - m.hb);
-  }
   return m;
-}
-
-__device__ __forceinline__ VMeta shfl_vmeta(const VMeta& m, int src) {
-  VMeta r;
-  r.b0 = __shfl_sync(FULL, m.b0, src);
-  r.b1 = __shfl_sync(FULL, m.b1, src);
-  r.hb = __shfl_sync(FULL, m.hb, src);
-  r.hT = __shfl_sync(FULL, m.hT, src);
-  r.hid = __shfl_sync(FULL, m.hid, src);
-  return r;
 }
 
 // The staged leaf set F of a level-(k-2) list: either materialised in this warp's shared
 // memory (sorted, every S[k-2]-independent filter applied), or -- when F is a window of a
-// single adjacency list N(y) with no per-element filter (lf_byref) and y has a bitmap or
-// hash set -- referenced in place: F = adj[offs[y] + a, offs[y] + b) and "w in F" is
-// "w in [F_min, F_max] and w in N(y)" by y's bitmap / hash set (no copy, no size cap).
+// single adjacency list N(y) with no per-element filter (lf_byref) and y has a hub bitmap --
+// referenced in place: F = adj[offs[y] + a, offs[y] + b) and "w in F" is "w in [F_min, F_max]
+// and w in N(y)" by y's bitmap (no copy, no size cap).
 struct FRef {
   const int* F;  // sorted ids F[0, nF) (shared or global memory)
-  int hid;       // by reference: y's bitmap row, -1 = none
-  long long hb;  // by reference: y's hash set slots [hb, hb + hT)
-  unsigned hT;   // 0 = none; hid < 0 && hT == 0 means F is materialised in shared memory
+  int hid;       // by reference: y's bitmap row; -1 = F is materialised in shared memory
   unsigned fix;  // by reference, plans without an N(S[k-2]) operand: lanes j whose S[j] must differ from
                  // the leaf's candidates (injectivity at positions <= k-3) and lies inside F
 };
@@ -462,121 +462,6 @@ __device__ __forceinline__ int fixed_in_window(const FRef& fr, int sreg, int lo,
     n += (s >= fmin && s <= fmax) ? 1 : 0;
   }
   return n;
-}
-
-// |{ v in L[s, e) : vmin <= v <= vmax, v in set }| for a sorted list L (global or shared
-// memory) and an O(1) probe set (bitmap row, else hash set).  Two 32-id batches per
-// round so that two probe loads per lane are in flight; stops past vmax.
-__device__ long long count_stream_probe(const KParams& P, const int* L, long long s, long long e, int vmin, int vmax,
-                                        int hid, long long hb, unsigned hT, int lane) {
-  const uint32_t* row = hid >= 0 ? P.hub_bits + (long long)hid * P.hub_words : nullptr;
-  long long total = 0;
-  for (long long base = s; base < e; base += 64) {
-    const long long i0 = base + lane, i1 = i0 + 32;
-    const int v0 = i0 < e ? L[i0] : INT_MAX, v1 = i1 < e ? L[i1] : INT_MAX;
-    const bool in0 = i0 < e && v0 >= vmin && v0 <= vmax;
-    const bool in1 = i1 < e && v1 >= vmin && v1 <= vmax;
-    bool ok0, ok1;
-    if (row) {
-      const uint32_t w0 = in0 ? __ldg(row + (v0 >> 5)) : 0u;
-      const uint32_t w1 = in1 ? __ldg(row + (v1 >> 5)) : 0u;
-      ok0 = (w0 >> (v0 & 31)) & 1u;
-      ok1 = (w1 >> (v1 & 31)) & 1u;
-    } else {
-      const unsigned s0 = hash_home(hT, v0), s1 = hash_home(hT, v1);
-      const int4 q0 = in0 ? __ldg(reinterpret_cast<const int4*>(P.hslots + hb + (s0 & ~3u))) : make_int4(0, 0, 0, -1);
-      const int4 q1 = in1 ? __ldg(reinterpret_cast<const int4*>(P.hslots + hb + (s1 & ~3u))) : make_int4(0, 0, 0, -1);
-      int r0 = in0 ? hash_group(q0, v0, s0 & 3u) : 0;
-      int r1 = in1 ? hash_group(q1, v1, s1 & 3u) : 0;
-      if (r0 < 0) r0 = hash_tail(P.hslots, hb, hT, v0, s0 & ~3u);
-      if (r1 < 0) r1 = hash_tail(P.hslots, hb, hT, v1, s1 & ~3u);
-      ok0 = r0 > 0;
-      ok1 = r1 > 0;
-    }
-    total += __popc(__ballot_sync(FULL, ok0)) + __popc(__ballot_sync(FULL, ok1));
-    if (__any_sync(FULL, (i1 < e ? v1 : (i0 < e ? v0 : INT_MIN)) > vmax)) break;
-  }
-  return total;
-}
-
-// lower_bound of v in F[lo, hi): shared-memory halving search, or a warp-cooperative
-// 32-ary search when F is referenced in global memory
-__device__ __forceinline__ int f_lower_bound(const FRef& fr, int lo, int hi, int v, int lane) {
-  if (fr.hid >= 0 || fr.hT) return lo + (int)warp_lower_bound(fr.F + lo, hi - lo, v, lane);
-  return smem_lower_bound(fr.F, lo, hi, v);
-}
-
-// Leaf of a count job with the staged set F[0, nF) (fr): |F ∩ window(x) ∩ N(x)| when N(x)
-// is an operand, else |F ∩ window(x)| minus x itself, where x = S[k-2] (DESIGN.md "leaf
-// staging"); mx = N(x)'s metadata (loaded in batches of 32 leaves by the caller).  A cost
-// model picks one of: stream F and probe N(x) (hub bitmap, else hash set, else per-lane
-// binary search with an advancing lower bound), or stream N(x) -- narrowed to
-// [F_min, F_max] by a warp-cooperative search -- and probe F (y's bitmap / hash set when
-// F is referenced, else a shared-memory binary search).
-template <bool STATS>
-__device__ long long leaf_staged(const KParams& P, Ctx<STATS>& c, const FRef& fr, int nF, int x, const VMeta& mx) {
-  const DevPlan& pl = P.plan;
-  const int lane = c.lane;
-  const int* F = fr.F;
-  const bool byref = fr.hid >= 0 || fr.hT;
-  int lo = 0, hi = nF;
-  if (pl.lf_lo_var) lo = f_lower_bound(fr, 0, nF, x + 1, lane);
-  if (pl.lf_hi_var) hi = f_lower_bound(fr, lo, nF, x, lane);
-  if (lo >= hi) return 0;
-  if (!pl.lf_var) {
-    long long cnt = hi - lo - fixed_in_window(fr, c.sreg, lo, hi);
-    if (pl.lf_inj_var) {
-      const int i = f_lower_bound(fr, lo, hi, x, lane);
-      cnt -= (i < hi && F[i] == x) ? 1 : 0;
-    }
-    return cnt;
-  }
-  const long long b0 = mx.b0, b1 = mx.b1;
-  const int hid = mx.hid;
-  const unsigned hT = mx.hT;
-  const long long a = hi - lo, b = b1 - b0;
-  if (b == 0) return 0;
-  // cost model in "dependent global load" units: stream F and probe N(x) costs
-  // ceil(a/32) rounds of one probe of N(x); streaming N(x) costs a window
-  // search plus ceil(b/32) rounds of one load and one probe of F
-  const int g = P.lf_cost_g;
-  const int lgb = 32 - __clz((int)min(b, (long long)INT_MAX));
-  const int lga = 32 - __clz((int)a);
-  const long long costA = ((a + 31) >> 5) * (long long)(hid >= 0 ? g : hT ? g + P.lf_cost_h : lgb * g);
-  const long long costB = 3ll * g + ((b + 31) >> 5) * (long long)(byref ? 2 * g + P.lf_cost_h : g + lga);
-  if (costA <= costB && (hid >= 0 || hT)) return count_stream_probe(P, F, lo, hi, INT_MIN, INT_MAX, hid, mx.hb, hT, lane);
-  long long total = 0;
-  if (costA <= costB) {
-    long long pb = b0;  // advancing lower bound into N(x)
-    for (int base = lo; base < hi; base += 32) {
-      const int i = base + lane;
-      const bool inr = i < hi;
-      const int v = inr ? F[i] : INT_MAX;
-      const int last_lane = min(31, hi - 1 - base);
-      int pos = (int)(b1 - pb);
-      if (inr) pos = lower_bound_dev(P.adj + pb, (int)(b1 - pb), v);
-      const bool ok = inr && pos < b1 - pb && __ldg(P.adj + pb + pos) == v;
-      pb += __shfl_sync(FULL, pos, last_lane);
-      total += __popc(__ballot_sync(FULL, ok));
-      if (pb >= b1) break;
-    }
-    return total;
-  }
-  const int fmin = F[lo], fmax = F[hi - 1];
-  const long long s = b0 + (b > 64 ? warp_lower_bound(P.adj + b0, b, fmin, lane) : 0);
-  if (byref) return count_stream_probe(P, P.adj, s, b1, fmin, fmax, fr.hid, fr.hb, fr.hT, lane);
-  for (long long sb = s; sb < b1; sb += 32) {
-    const long long i = sb + lane;
-    const int v = i < b1 ? __ldg(P.adj + i) : INT_MAX;
-    bool ok = v >= fmin && v <= fmax;
-    if (ok) {
-      const int j = smem_lower_bound(F, lo, hi, v);
-      ok = F[j] == v;  // j < hi since v <= fmax
-    }
-    total += __popc(__ballot_sync(FULL, ok));
-    if (__shfl_sync(FULL, v, 31) >= fmax) break;
-  }
-  return total;
 }
 
 // per-lane lower_bound of v in the sorted F[lo, hi) (shared or global memory)
@@ -599,21 +484,48 @@ __device__ __forceinline__ int warp_excl_scan(int v, int lane) {
   return x - v;
 }
 
+// Branch-free lower_bound of four values in the same sorted list L[lo, lo + n) (global, shared
+// or generic memory): every step issues the four probes together (independent loads in flight)
+// and all four share the trip count ceil(log2 n).  Results in r0..r3 (indices into L).
+__device__ __forceinline__ void lower_bound4(const int* L, int lo, int n, int v0, int v1, int v2, int v3, int& r0,
+                                             int& r1, int& r2, int& r3) {
+  r0 = r1 = r2 = r3 = lo;
+  if (n <= 0) return;
+  while (n > 1) {
+    const int half = n >> 1;
+    const int a0 = L[r0 + half], a1 = L[r1 + half], a2 = L[r2 + half], a3 = L[r3 + half];
+    r0 = a0 < v0 ? r0 + half : r0;
+    r1 = a1 < v1 ? r1 + half : r1;
+    r2 = a2 < v2 ? r2 + half : r2;
+    r3 = a3 < v3 ? r3 + half : r3;
+    n -= half;
+  }
+  r0 += L[r0] < v0;
+  r1 += L[r1] < v1;
+  r2 += L[r2] < v2;
+  r3 += L[r3] < v3;
+}
+
+__device__ __forceinline__ unsigned bit_of(const uint32_t* row, int v) { return (__ldg(row + (v >> 5)) >> (v & 31)) & 1u; }
+
 // A whole batch of nb <= 32 staged leaves at once: lane j
 // holds leaf x_j = S[k-2] and N(x_j)'s metadata.  The count is only summed, so the batch's
-// work is flattened into two load-balanced streams of (leaf, element) pairs:
+// work is flattened into two load-balanced streams over the leaves' elements:
 //   A: leaves where streaming F is cheaper: elements F[lo_j .. hi_j), each probed in N(x_j)
 //      (hub bitmap, else binary search);
-//   B: the others: elements of N(x_j), each tested against [F_min_j, F_max_j] and probed in
-//      F (y's bitmap / hash set when F is referenced, else a shared-memory binary search).
-// Every lane takes one pair per round whatever the leaves' sizes -- no per-leaf rounds.
+//   B: the others: elements of N(x_j) narrowed to [F_min_j, F_max_j], each probed in F (y's
+//      bitmap when F is referenced, else a shared-memory binary search).
+// Both streams are walked in aligned 16-byte groups: one 128-bit load gives a lane four
+// consecutive ids of one leaf (north_star "vectorised coalesced 128-bit adjacency loads"),
+// whose four probes are then issued together.  A lane moves to the next leaf by walking the
+// batch's prefix sums in shared memory; hits are summed per lane and reduced once per batch.
 template <bool STATS>
 __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr, int nF, int nb, int x,
                                 const VMeta& m) {
   const DevPlan& pl = P.plan;
   const int lane = c.lane;
   const int* F = fr.F;
-  const bool byref = fr.hid >= 0 || fr.hT;
+  const bool byref = fr.hid >= 0;
   const bool act = lane < nb;
   int lo = 0, hi = nF;
   if (act && pl.lf_lo_var) lo = lane_lower_bound(F, 0, nF, x + 1);
@@ -624,7 +536,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     if (cnt && pl.lf_inj_var) {  // x itself inside F[lo, hi)?
       if (fr.hid >= 0) {            // referenced F of a hub y: range test + one bitmap load
         cnt -= (x >= F[lo] && x <= F[hi - 1] &&
-                ((__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (x >> 5)) >> (x & 31)) & 1u)) ? 1 : 0;
+                bit_of(P.hub_bits + (long long)fr.hid * P.hub_words, x)) ? 1 : 0;
       } else {
         const int i = lane_lower_bound(F, lo, hi, x);
         cnt -= (i < hi && F[i] == x) ? 1 : 0;
@@ -633,101 +545,139 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
     return cnt;
   }
+  // F is walked from its 16-byte aligned base: F = Fal + fo
+  const int fo = (int)((reinterpret_cast<uintptr_t>(F) >> 2) & 3u);
+  const int* const Fal = F - fo;
   const int a = (act && lo < hi) ? hi - lo : 0;
-  const int b = act ? (int)(m.b1 - m.b0) : 0;
-  int wA = 0, wB = 0;
-  if (a > 0 && b > 0) {
-    const int lgb = 32 - __clz(b), lga = 32 - __clz(a);
-    const long long uA = m.hid >= 0 ? P.ua_hub : 3 + lgb;
-    const long long uB = byref ? (fr.hid >= 0 ? P.ub_ref : P.ub_ref + P.lf_cost_h) : 3 + (lga >> 1);
-    if ((long long)a * uA <= (long long)b * uB) wA = a;
-    else wB = b;
+  int bs = 0, be = act ? (int)(m.b1 - m.b0) : 0;
+  int gA = 0, gB = 0;  // this leaf's 16-byte groups in stream A / B
+  if (a > 0 && be > 0) {
+    // N(x) narrowed to [F_min, F_max] (both bounds by search for long lists)
+    if (be >= 64) {
+      const int* N = P.adj + m.b0;
+      bs = lower_bound_dev(N, be, F[lo]);
+      be = bs + lower_bound_dev(N + bs, be - bs, F[hi - 1] + 1);
+    }
+    const int b = be - bs;
+    if (b > 0) {
+      const int lgb = 32 - __clz(be), lga = 32 - __clz(a);
+      const long long uA = m.hid >= 0 ? kUaHub : 3 + lgb;
+      const long long uB = byref ? kUbRef : 3 + (lga >> 1);
+      if ((long long)a * uA <= (long long)b * uB) gA = ((fo + hi + 3) >> 2) - ((fo + lo) >> 2);
+      else gB = (int)(((m.b0 + be + 3) >> 2) - ((m.b0 + bs) >> 2));
+    }
   }
-  // the batch's per-leaf entries go to shared memory: a lane then reads its current leaf's
-  // entry only when it moves to the next leaf (no warp-wide shuffles per element)
-  // shared-window addresses derived from tdfs_smem (32-bit LDS/STS, cheap to recompute)
   char* const wbase = reinterpret_cast<char*>(tdfs_smem) + P.meta_off + (int)(threadIdx.x >> 5) * kMetaBytesPerWarp;
   LeafMeta* meta = reinterpret_cast<LeafMeta*>(wbase);
   int* pre = reinterpret_cast<int*>(wbase + 32 * sizeof(LeafMeta));
   if (act) {
     LeafMeta e;
     e.b0 = m.b0;
-    e.deg = b;
+    e.deg = (int)(m.b1 - m.b0);
     e.hid = m.hid;
-    e.lo = lo;
-    e.hi = hi;
+    e.lo = gA ? bs : lo;  // A: the narrowed N(x) range [bs, be) searched; B: the F window
+    e.hi = gA ? be : hi;
+    e.s = gA ? fo + lo : bs;
+    e.e = gA ? fo + hi : be;
     meta[lane] = e;
   }
-  long long total = 0;
-  // stream A: (j, F[lo_j + i]) probed in N(x_j)
+  unsigned cnt = 0;
+  // stream A: F elements of leaf j probed in N(x_j)
   {
-    const int p = warp_excl_scan(wA, lane);
-    const int tot = __shfl_sync(FULL, p + wA, 31);
+    const int p = warp_excl_scan(gA, lane);
+    const int tot = __shfl_sync(FULL, p + gA, 31);
     __syncwarp();
     pre[lane] = act ? p : tot;
     if (lane == 0) pre[32] = tot;
     __syncwarp();
-    int j = -1, jn = 0, pj = 0, lj = 0, hidj = -1, degj = 0, pb = 0;
+    int j = -1, jn = 0, pj = 0, g0 = 0, sj = 0, ej = 0, hidj = -1, degj = 0, pb = 0;
     long long b0j = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
-      bool ok = false;
       if (idx < tot) {
         if (idx >= jn) {  // move to the leaf holding idx (per lane, shared-memory reads)
           do { ++j; jn = pre[j + 1]; } while (jn <= idx);
           pj = pre[j];
           const LeafMeta e = meta[j];
-          lj = e.lo; hidj = e.hid; degj = e.deg; b0j = e.b0;
-          pb = 0;
+          sj = e.s; ej = e.e; hidj = e.hid; b0j = e.b0;
+          pb = e.lo;  // N(x_j)[lo, hi) holds every id in [F_min_j, F_max_j]
+          degj = e.hi;
+          g0 = sj >> 2;
         }
-        const int w = F[lj + idx - pj];
+        const int g = g0 + idx - pj;
+        const int4 q = *reinterpret_cast<const int4*>(Fal + 4 * g);
+        const int i0 = 4 * g;
+        const bool k0 = i0 >= sj && i0 < ej, k1 = i0 + 1 >= sj && i0 + 1 < ej;
+        const bool k2 = i0 + 2 >= sj && i0 + 2 < ej, k3 = i0 + 3 >= sj && i0 + 3 < ej;
         if (hidj >= 0) {
-          ok = (__ldg(P.hub_bits + (long long)hidj * P.hub_words + (w >> 5)) >> (w & 31)) & 1u;
+          const uint32_t* row = P.hub_bits + (long long)hidj * P.hub_words;
+          cnt += (k0 ? bit_of(row, q.x) : 0u) + (k1 ? bit_of(row, q.y) : 0u) + (k2 ? bit_of(row, q.z) : 0u) +
+                 (k3 ? bit_of(row, q.w) : 0u);
         } else {
-          // this lane's ids of one leaf increase round by round: search N(x_j) from the last hit
-          pb += lower_bound_dev(P.adj + b0j + pb, degj - pb, w);
-          ok = pb < degj && __ldg(P.adj + b0j + pb) == w;
+          // this lane's ids of one leaf increase group by group: search N(x_j) from the last hit;
+          // ids outside the leaf's window search as +inf (they sit past every valid id)
+          const int v0 = k0 ? q.x : INT_MAX, v1 = k1 ? q.y : INT_MAX, v2 = k2 ? q.z : INT_MAX, v3 = k3 ? q.w : INT_MAX;
+          const int* N = P.adj + b0j;
+          int r0, r1, r2, r3;
+          lower_bound4(N, pb, degj - pb, v0, v1, v2, v3, r0, r1, r2, r3);
+          cnt += (k0 && r0 < degj && N[r0] == v0) + (k1 && r1 < degj && N[r1] == v1) +
+                 (k2 && r2 < degj && N[r2] == v2) + (k3 && r3 < degj && N[r3] == v3);
+          pb = k0 ? r0 : pb;
+          pb = k1 ? r1 : pb;
+          pb = k2 ? r2 : pb;
+          pb = k3 ? r3 : pb;
         }
       }
-      total += __popc(__ballot_sync(FULL, ok));
     }
   }
-  // stream B: (j, N(x_j)[i]) tested against F
+  // stream B: N(x_j) elements inside [F_min_j, F_max_j] probed in F
   {
-    const int p = warp_excl_scan(wB, lane);
-    const int tot = __shfl_sync(FULL, p + wB, 31);
+    const int p = warp_excl_scan(gB, lane);
+    const int tot = __shfl_sync(FULL, p + gB, 31);
     __syncwarp();
     pre[lane] = act ? p : tot;
     if (lane == 0) pre[32] = tot;
     __syncwarp();
+    const int4* const adj4 = reinterpret_cast<const int4*>(P.adj);
+    const uint32_t* const frow = fr.hid >= 0 ? P.hub_bits + (long long)fr.hid * P.hub_words : nullptr;
     int j = -1, jn = 0, pj = 0, loj = 0, hij = 0, fminj = 0, fmaxj = 0;
-    long long b0j = 0;
+    long long g0 = 0, sj = 0, ej = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
-      bool ok = false;
       if (idx < tot) {
         if (idx >= jn) {
           do { ++j; jn = pre[j + 1]; } while (jn <= idx);
           pj = pre[j];
           const LeafMeta e = meta[j];
-          loj = e.lo; hij = e.hi; b0j = e.b0;
+          loj = e.lo; hij = e.hi;
+          sj = e.b0 + e.s;
+          ej = e.b0 + e.e;
+          g0 = sj >> 2;
           fminj = F[loj];
           fmaxj = F[hij - 1];
         }
-        const int v = __ldg(P.adj + b0j + idx - pj);
-        if (v >= fminj && v <= fmaxj) {
-          if (fr.hid >= 0) ok = (__ldg(P.hub_bits + (long long)fr.hid * P.hub_words + (v >> 5)) >> (v & 31)) & 1u;
-          else if (fr.hT) ok = hash_contains(P.hslots, fr.hb, fr.hT, v);
-          else ok = F[smem_lower_bound(F, loj, hij, v)] == v;  // index < hij since v <= F[hij - 1]
+        const long long g = g0 + idx - pj;
+        const int4 q = __ldg(adj4 + g);
+        const long long i0 = g << 2;
+        const bool k0 = i0 >= sj && i0 < ej && q.x >= fminj && q.x <= fmaxj;
+        const bool k1 = i0 + 1 >= sj && i0 + 1 < ej && q.y >= fminj && q.y <= fmaxj;
+        const bool k2 = i0 + 2 >= sj && i0 + 2 < ej && q.z >= fminj && q.z <= fmaxj;
+        const bool k3 = i0 + 3 >= sj && i0 + 3 < ej && q.w >= fminj && q.w <= fmaxj;
+        if (frow) {
+          cnt += (k0 ? bit_of(frow, q.x) : 0u) + (k1 ? bit_of(frow, q.y) : 0u) + (k2 ? bit_of(frow, q.z) : 0u) +
+                 (k3 ? bit_of(frow, q.w) : 0u);
+        } else {
+          // F in shared memory: four lockstep searches; a kept id is <= F_max so its index is < hi
+          int r0, r1, r2, r3;
+          lower_bound4(F, loj, hij - loj, q.x, q.y, q.z, q.w, r0, r1, r2, r3);
+          cnt += (k0 && F[r0] == q.x) + (k1 && F[r1] == q.y) + (k2 && F[r2] == q.z) + (k3 && F[r3] == q.w);
         }
       }
-      total += __popc(__ballot_sync(FULL, ok));
     }
   }
   __syncwarp();
-  return total;
+  return (long long)__reduce_add_sync(FULL, cnt);
 }
-
 // Stage F for the level-(k-2) list just built (see FRef).  Returns |F|, or -2 when F
 // would have to be materialised and exceeds the shared-memory stage (generic per leaf).
 template <bool STATS>
@@ -736,13 +686,11 @@ __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& 
   const int lane = c.lane;
   fr.F = c.sF;
   fr.hid = -1;
-  fr.hb = 0;
-  fr.hT = 0;
   fr.fix = 0;
-  if (pl.lf_byref && P.lf_byref) {
+  if (pl.lf_byref) {
     const int y = getS(c.sreg, __ffs(pl.bwd[kVF]) - 1);
     const VMeta my = load_vmeta(P, y);
-    if (my.hid >= 0 || my.hT) {
+    if (my.hid >= 0) {
       const uint32_t lom = pl.lo_mask[kVF], him = pl.hi_mask[kVF];
       const int wlo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
       const int whi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
@@ -752,16 +700,11 @@ __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& 
       const long long b = whi < INT_MAX ? a + warp_lower_bound(P.adj + my.b0 + a, n - a, whi, lane) : n;
       fr.F = P.adj + my.b0 + a;
       fr.hid = my.hid;
-      fr.hb = my.hb;
-      fr.hT = my.hT;
       if (const uint32_t im = pl.inj_mask[kVF]) {  // matched S[j] (j <= k-3) that lie inside F
         bool in = false;
         if ((im >> lane) & 1u) {
           const int s = c.sreg;
-          if (s >= wlo && s < whi) {
-            if (my.hid >= 0) in = (__ldg(P.hub_bits + (long long)my.hid * P.hub_words + (s >> 5)) >> (s & 31)) & 1u;
-            else in = hash_contains(P.hslots, my.hb, my.hT, s);
-          }
+          if (s >= wlo && s < whi) in = bit_of(P.hub_bits + (long long)my.hid * P.hub_words, s);
         }
         fr.fix = __ballot_sync(FULL, in);
       }
@@ -802,7 +745,7 @@ __device__ bool split_level2_ranges(const KParams& P, Ctx<STATS>& c, const Queue
   const int lane = c.lane;
   const uint32_t* table = c.tables;  // level index 0 = position 2
   const int rem = size - from;
-  const int g = max(P.range_min, (rem + P.range_maxt - 1) / P.range_maxt);
+  const int g = max(kRangeMin, (rem + kRangeMaxT - 1) / kRangeMaxT);
   const int ntask = (rem + g - 1) / g;
   const int i0 = from + lane * g, i1 = i0 + g;
   int lo = 0, hi = c.w2hi;
@@ -859,7 +802,7 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         if (STATS && lane == 0) c.touts++;
         if (k == 4 && P.range_split && P.range_ok) {
           // <= 32 remaining siblings finish in place (tasks strictly shrink: progress at tau = 0)
-          if (size - it <= P.range_min) {
+          if (size - it <= kRangeMin) {
             if (lane == 0) c.t0 = globaltimer();
             grace = true;
             continue;
@@ -890,13 +833,9 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         // loaded by one lane each (independent loads), then each leaf is one |F ∩ N(x)|
         const int nb = min(32, size - it);
         const int vl = lane < nb ? paged_read(P, table, it + lane) : 0;
-        VMeta ml = {0, 0, 0, 0u, -1};
+        VMeta ml = {0, 0, -1};
         if (lane < nb) ml = load_vmeta(P, vl);
-        long long n = 0;
-        if (P.leaf_flat) n = leaf_batch(P, c, fr, nF, nb, vl, ml);
-        else
-          for (int j = 0; j < nb; j++) n += leaf_staged(P, c, fr, nF, __shfl_sync(FULL, vl, j), shfl_vmeta(ml, j));
-        c.count += (unsigned long long)n;
+        c.count += (unsigned long long)leaf_batch(P, c, fr, nF, nb, vl, ml);
         if (lane == d) c.liter = it + nb;
         continue;
       }
@@ -936,7 +875,8 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
     int v0 = 0, v1 = 0;
     bool ok = inr;
     if (inr) {
-      const long long e = (long long)P.shard_rank + j * (long long)P.shard_world;
+      const long long e = P.task_edges ? (long long)__ldg(P.task_edges + j)
+                                       : (long long)P.shard_rank + j * (long long)P.shard_world;
       v0 = __ldg(P.src + e);
       v1 = __ldg(P.adj + e);
       if (pl.edge_cons == 1) ok = v0 < v1;
@@ -1000,7 +940,7 @@ template <int MODE, bool STATS>
 #ifndef TDFS_MIN_BLOCKS
 #define TDFS_MIN_BLOCKS 12  // 40 registers: measured best of 8..16 on config 2
 #endif
-__global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParams P) {
+__global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(const KParams P) {
   const int lane = threadIdx.x & 31;
   const long long gwarp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   Ctx<STATS> c;
@@ -1020,7 +960,7 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
   c.sF = tdfs_smem + (threadIdx.x >> 5) * P.fcap;
   const Queue q = make_queue(P);
   int* active = reinterpret_cast<int*>(ctr(P, C_ACTIVE));
-  unsigned long long* cursor = ctr(P, C_CURSOR);
+  unsigned long long* cursor = P.gcursor;
 
   if (lane == 0) atomicAdd(active, 1);
   bool busy = true;
@@ -1066,7 +1006,7 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
       if (range) {
         c.w2lo = t3;
         c.w2hi = t4;
-        c.w2mode = P.range_mode ? P.range_mode : (P.reuse2_used ? 2 : 1);
+        c.w2mode = P.reuse2_used ? 2 : 1;
       }
       const bool ok = dfs<MODE, STATS>(P, c, q, (t3 == -2 || range) ? 2 : 3);
       c.w2lo = 0;
@@ -1082,7 +1022,12 @@ __global__ void __launch_bounds__(128, TDFS_MIN_BLOCKS) tdfs_kernel(const KParam
     // 2. next chunk of initial edge tasks
     long long j0 = P.n_tasks;
     if (lane == 0) {
-      if ((long long)ld_relaxed_s64(cursor) < P.n_tasks) {
+      if (P.gshared) {  // cursor shared with other ranks / GPUs (NEXT-3): system-scope atomics
+        if (ld_relaxed_sys_s64(cursor) < P.n_tasks) {
+          j0 = (long long)atomicAdd_system(cursor, (unsigned long long)P.chunk);
+          c.t0 = globaltimer();
+        }
+      } else if ((long long)ld_relaxed_s64(cursor) < P.n_tasks) {
         j0 = (long long)atomicAdd(cursor, (unsigned long long)P.chunk);
         c.t0 = globaltimer();
       }
@@ -1176,7 +1121,8 @@ int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, pick_kernel(enumerate ? 1 : 0, stats), wpb * 32,
                                                                 smem_bytes(wpb, fcap));
   if (e != cudaSuccess) return cuda_fail(e, "occupancy");
-  *out = std::max(1, nb);
+  if (nb < 1) return fail(TDFS_E_INVALID_ARG, "occupancy: the kernel cannot be resident with this block shape");
+  *out = nb;
   return TDFS_OK;
 }
 
@@ -1195,10 +1141,14 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return cuda_fail(e, "device attribute");
   L->wpb = o->warps_per_block > 0 ? o->warps_per_block : 4;
-  if (L->wpb > 32) return fail(TDFS_E_INVALID_ARG, "opts.warps_per_block must be <= 32");
+  if (L->wpb > kBlockThreads / 32)  // the kernel's __launch_bounds__
+    return fail(TDFS_E_INVALID_ARG, "opts.warps_per_block must be <= " + std::to_string(kBlockThreads / 32));
+  if (o->shard_policy != TDFS_SHARD_ROUND_ROBIN && o->shard_policy != TDFS_SHARD_DEGREE_BALANCED)
+    return fail(TDFS_E_INVALID_ARG, "opts.shard_policy");
+  if (o->reserved_ != 0) return fail(TDFS_E_INVALID_ARG, "opts.reserved_ must be 0");
+  if (o->shared_cursor && (reinterpret_cast<uintptr_t>(o->shared_cursor) & 7u))
+    return fail(TDFS_E_INVALID_ARG, "opts.shared_cursor must be 8-byte aligned");
   L->fcap = kLeafStage;
-  if (const char* e = getenv("TDFS_FCAP")) L->fcap = atoi(e);  // tuning knob (experiments)
-  if (L->fcap < 0 || L->fcap > 8192) return fail(TDFS_E_INVALID_ARG, "TDFS_FCAP must be in [0, 8192]");
   if (o->blocks > 0) {
     L->blocks = o->blocks;
   } else {
@@ -1291,6 +1241,20 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.shard_rank = o->shard_rank;
   P.shard_world = o->shard_world;
   P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
+  P.gcursor = (unsigned long long*)(base + L.ctr) + C_CURSOR * kCounterStride;
+  if (o->shared_cursor) {
+    // cross-rank dynamic balancing (NEXT-3): every directed edge, chunks from the shared cursor
+    P.shard_rank = 0;
+    P.shard_world = 1;
+    P.n_tasks = g->nnz;
+    P.gcursor = reinterpret_cast<unsigned long long*>(o->shared_cursor);
+    P.gshared = 1;
+  } else if (o->shard_world > 1 && o->shard_policy == TDFS_SHARD_DEGREE_BALANCED) {
+    int64_t nt = 0;
+    if ((rc = shard_task_list(g, o->shard_rank, o->shard_world, o->shard_policy, &P.task_edges, &nt)) != TDFS_OK)
+      return rc;
+    P.n_tasks = nt;
+  }
   P.chunk = o->chunk;
   P.n_levels = L.n_levels;
   P.slots = (QSlot*)(base + L.slots);
@@ -1307,43 +1271,12 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
   P.meta_off = (int)smem_meta_offset(L.wpb, L.fcap);
-  P.lf_cost_g = 6;
-  P.lf_cost_h = 2;
-  P.ua_hub = 4;
-  P.ub_ref = 4;
-  if (const char* e = getenv("TDFS_UA_HUB")) P.ua_hub = atoi(e);  // tuning knobs (experiments)
-  if (const char* e = getenv("TDFS_UB_REF")) P.ub_ref = atoi(e);
-  if (const char* e = getenv("TDFS_LF_HCOST")) P.lf_cost_h = atoi(e);  // tuning knob (experiments)
-  P.range_split = 1;
-  P.range_min = 32;
-  P.range_maxt = 32;
-  if (const char* e = getenv("TDFS_RANGE_MIN")) P.range_min = std::max(1, atoi(e));  // tuning knobs (experiments)
-  if (const char* e = getenv("TDFS_RANGE_MAXT")) P.range_maxt = std::min(32, std::max(2, atoi(e)));
-  if (const char* e = getenv("TDFS_RANGE_MODE")) P.range_mode = atoi(e);
-  if (const char* e = getenv("TDFS_RANGE_FORCE")) P.range_ok = atoi(e);
-  if (const char* e = getenv("TDFS_RANGE_SPLIT")) P.range_split = atoi(e);  // tuning knob (experiments)
-  P.leaf_flat = 1;
-  if (const char* e = getenv("TDFS_LEAF_FLAT")) P.leaf_flat = atoi(e);  // tuning knob (experiments)
-  P.lf_byref = 1;
-  if (const char* e = getenv("TDFS_BYREF")) P.lf_byref = atoi(e);  // tuning knob (experiments)
-  P.coop_window = 1;
-  if (const char* e = getenv("TDFS_COOP")) P.coop_window = atoi(e);  // tuning knob (experiments)
-  if (const char* e = getenv("TDFS_LF_COST")) P.lf_cost_g = atoi(e);  // tuning knob (experiments)
-  P.merge_ratio = kMergeRatio;
-  if (const char* e = getenv("TDFS_MERGE_RATIO")) P.merge_ratio = atoi(e);  // tuning knob (experiments)
-  P.merge_ratio_hash = kMergeRatioHash;
-  if (const char* e = getenv("TDFS_MERGE_RATIO_H")) P.merge_ratio_hash = atoi(e);  // tuning knob (experiments)
-  P.bsearch_variant = 0;
+  P.range_split = (o->flags & TDFS_RUN_NO_RANGE_TASKS) ? 0 : 1;
   if (g->d_hub_bits && !(o->flags & TDFS_RUN_NO_HUB_BITMAP)) {
     P.hub_id = g->d_hub_id;
     P.hub_bits = g->d_hub_bits;
     P.hub_words = g->hub_words;
   }
-  if (g->d_hslots && !(o->flags & TDFS_RUN_NO_HASH)) {
-    P.hoff = g->d_hoff;
-    P.hslots = g->d_hslots;
-  }
-  if (const char* e = getenv("TDFS_BSEARCH")) P.bsearch_variant = atoi(e);
   P.out = d_out;
   P.cap = cap;
   int32_t* d_trace = nullptr;

@@ -144,9 +144,21 @@ void build_dev(const QueryAdj& q, Plan& P) {
       if (d.deg_min[r] > std::max(d.deg_min[p], nb)) continue;
       if ((d.lo_mask[r] & d.lo_mask[p]) != d.lo_mask[r]) continue;
       if ((d.hi_mask[r] & d.hi_mask[p]) != d.hi_mask[r]) continue;
+      d.src_mask[p] |= 1u << r;
       if (best < 0 || __builtin_popcount(d.bwd[r]) >= __builtin_popcount(d.bwd[best])) best = r;
     }
     d.reuse[p] = (int8_t)best;
+  }
+  // R32 count-only last position (for the roofline bytes, independent of which r is reused)
+  if (q.k >= 3) {
+    const int p = q.k - 1;
+    const bool nolab = d.label[p] < 0, nodeg = d.deg_min[p] == 0;
+    bool co = __builtin_popcount(d.bwd[p]) == 1 && nolab && nodeg;
+    for (int r = 2; r < p; r++)
+      if (((d.src_mask[p] >> r) & 1u) && d.bwd[r] == d.bwd[p] && (nolab || d.label[r] == d.label[p]) &&
+          (nodeg || d.deg_min[r] >= d.deg_min[p]))
+        co = true;
+    d.cnt_only[p] = co;
   }
   // Count-only last position: when one list remains (one backward operand, or a reused C(r)
   // with B(r) = B(p)) and no per-element label/degree test is needed, |C(p)| is the size of

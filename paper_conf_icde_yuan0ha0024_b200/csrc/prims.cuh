@@ -4,8 +4,6 @@
 #pragma once
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr long long kMergeRatio = 4;  // Eq. (1) probe: merge when |B| <= 4 |A remaining|, else binary search
-constexpr int kMergeRatioHash = 1;    // ... and when |B| <= 1 |A remaining| if B has a hash set, else hash probes
 constexpr uint32_t NULL_PAGE = 0xffffffffu;
 constexpr int ERR_STACK = 1;
 
@@ -26,6 +24,11 @@ __device__ __forceinline__ void st_release_u32(unsigned* p, unsigned v) {
 __device__ __forceinline__ long long ld_relaxed_s64(const unsigned long long* p) {
   long long v;
   asm volatile("ld.relaxed.gpu.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ long long ld_relaxed_sys_s64(const unsigned long long* p) {
+  long long v;
+  asm volatile("ld.relaxed.sys.global.s64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
 __device__ __forceinline__ int ld_relaxed_s32(const int* p) {
@@ -66,44 +69,6 @@ __device__ __forceinline__ int lower_bound_dev(const int32_t* __restrict__ B, in
     }
   }
   return base;
-}
-
-// w in N(v) by v's adjacency hash set (graph.cu build_hash_index): T_v = T > 0 slots at
-// slots[h0 ..), w at or after its home slot, linear probing, EMPTY = -1.  Reads aligned
-// 16-byte groups of 4 slots; an EMPTY at or after the home slot ends a miss.
-__device__ __forceinline__ unsigned hash_home(unsigned T, int w) {
-  return ((unsigned)w * 2654435769u) >> (__clz(T) + 1);  // >> (32 - log2 T)
-}
-// one group: 1 = hit, 0 = miss, -1 = undecided (group full, no hit)
-__device__ __forceinline__ int hash_group(const int4 q, int w, unsigned skip) {
-  if (q.x == w || q.y == w || q.z == w || q.w == w) return 1;
-  const bool empty = (skip < 1 && q.x < 0) || (skip < 2 && q.y < 0) || (skip < 3 && q.z < 0) || q.w < 0;
-  return empty ? 0 : -1;
-}
-// continue a probe at group g (after an undecided group)
-__device__ __noinline__ bool hash_tail(const int32_t* __restrict__ slots, long long h0, unsigned T, int w, unsigned g) {
-  for (;;) {
-    g = (g + 4) & (T - 1);
-    const int r = hash_group(__ldg(reinterpret_cast<const int4*>(slots + h0 + g)), w, 0);
-    if (r >= 0) return r != 0;
-  }
-}
-__device__ __forceinline__ bool hash_contains(const int32_t* __restrict__ slots, long long h0, unsigned T, int w) {
-  const unsigned s = hash_home(T, w);
-  const int r = hash_group(__ldg(reinterpret_cast<const int4*>(slots + h0 + (s & ~3u))), w, s & 3u);
-  if (r >= 0) return r != 0;
-  return hash_tail(slots, h0, T, w, s & ~3u);
-}
-
-// Same result with power-of-two steps (trip count depends only on n: no divergence).
-__device__ __forceinline__ int lower_bound_pow2(const int32_t* __restrict__ B, int n, int v) {
-  if (n <= 0) return 0;
-  int pos = 0;
-  for (int step = 1 << (31 - __clz(n)); step > 0; step >>= 1) {
-    const int q = pos + step;
-    if (q <= n && __ldg(B + q - 1) < v) pos = q;
-  }
-  return pos;
 }
 
 // ------------------------------------------------------------ Q_task (Alg. 3)

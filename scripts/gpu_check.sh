@@ -1,12 +1,15 @@
 #!/bin/bash
-# One GPU round-trip: full -m gpu suite, then a bench line (no cpu baseline).
+# One GPU round-trip: the -m gpu suite (all failures listed), then a bench line.
+#   gpu_check.sh TAG [pytest -k expr]
 export PYTHONPATH=$PWD
 TAG=${1:-x}
-timeout 1500 python -m pytest tests -m gpu -q -x --timeout 400 --timeout-method=thread -p no:cacheprovider 2>&1 \
-  | grep -v "^  File\|^    " | tail -25 > gpurun_out/gputests_${TAG}.log
-cat gpurun_out/gputests_${TAG}.log
+K=${2:-}
+mkdir -p gpurun_out
+timeout 1800 python -m pytest tests -m gpu -q ${K:+-k "$K"} --timeout 600 --timeout-method=thread -p no:cacheprovider 2>&1 \
+  | grep -v "^  File\|^    " | tail -40 > gpurun_out/gputests_${TAG}.log
+tail -40 gpurun_out/gputests_${TAG}.log
 timeout 900 python bench.py --steps 3 --warmup 3 --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
-tail -2 gpurun_out/bench_${TAG}.err
+tail -3 gpurun_out/bench_${TAG}.err
 python - <<PY
 import json
 d = json.load(open("gpurun_out/bench_${TAG}.json"))

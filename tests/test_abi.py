@@ -43,7 +43,7 @@ def test_library_is_sm100a():
 
 
 def test_abi_version_and_status_strings():
-    assert M.tdfs_abi_version() == 1
+    assert M.tdfs_abi_version() == 2
     assert M.tdfs_status_string(0) == "TDFS_OK"
     assert M.tdfs_status_string(8) == "TDFS_E_STACK_EXHAUSTED"
     o = M.default_opts()

@@ -117,21 +117,21 @@ def test_split_counts_are_tau_invariant_on_skewed_graph():
             assert st["tasks_enqueued"] > 0 and st["tasks_enqueued"] == st["tasks_dequeued"]
 
 
-@pytest.mark.parametrize("range_split,force", [("1", None), ("1", "1"), ("0", None)])
-def test_level2_range_tasks_k4(monkeypatch, range_split, force):
+@pytest.mark.parametrize("range_split", [True, False])
+def test_level2_range_tasks_k4(range_split):
     """k = 4: a timed-out level-2 list is split into <= 32 id-range tasks <S0, S1, lo, hi>
      instead of one task per sibling.  With tau = 0 every level-2
     step splits; counts, per-level node counts and W (STATS variant) still equal the
     oracle's, and every pushed task is dequeued exactly once."""
-    monkeypatch.setenv("TDFS_RANGE_SPLIT", range_split)
-    if force:  # range tasks also where the planner's heuristic prefers per-sibling tasks (k4)
-        monkeypatch.setenv("TDFS_RANGE_FORCE", force)
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    fl = 0 if range_split else M.TDFS_RUN_NO_RANGE_TASKS
     g = T.rmat(11, 12, 4)
     for name in ("c4", "diamond", "k4", "tailed_triangle"):
         q = T.query(name)
         order = O.oracle_order(q)
         r = O.match(g, q, "auto", order=order, deg_filter=True, threads=8)
-        for kw in (dict(tau_ms=0.0), dict(tau_ms=0.0, blocks=2, warps_per_block=2), dict(tau_ms=0.01)):
+        for kw in (dict(tau_ms=0.0, flags=fl), dict(tau_ms=0.0, blocks=2, warps_per_block=2, flags=fl),
+                   dict(tau_ms=0.01, flags=fl)):
             cnt, st = U.count(g, q, "auto", order=order, stats=True, **kw)
             assert cnt == r["count"], (name, kw)
             assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k], (name, kw)

@@ -201,25 +201,26 @@ def test_hub_bitmaps_do_not_change_results():
         assert U.count(g, q, "auto") == U.count(g, q, "auto", flags=M.TDFS_RUN_NO_HUB_BITMAP | 4 | 8), name
 
 
-def test_hash_index_does_not_change_results(monkeypatch):
-    """Per-vertex adjacency hash sets replace binary searches of
-    non-hub operands; counts equal the oracle with the index on (default threshold and
-    every vertex hashed), off (TDFS_RUN_NO_HASH) and with hubs probed by hash too."""
+def test_leaf_set_paths_do_not_change_results():
+    """The staged leaf set F is referenced in place when its list
+    has a hub bitmap, materialised in shared memory otherwise, and -- when a materialised F
+    would exceed the 512-id stage -- replaced by Eq. (1) per leaf.  The same graph loaded with
+    hub bitmaps (default), without (hub_bitmap_bytes = -1: every F materialised, lists of
+    degree > 512 take the fallback) and with a 1-hub budget gives the oracle's counts for every
+    query shape whose last position is leaf-staged, with the leaf stage on and off."""
     import paper_conf_icde_yuan0ha0024_b200 as M
-    g = T.rmat(10, 16, 6)
-    assert int(np.bincount(g.edges.reshape(-1)).max()) >= 256  # hubs (bitmaps) and hashed lists both occur
-    names = ["triangle", "c4", "diamond", "tailed_triangle", "k4", "house"]
+    g = T.rmat(11, 24, 6)
+    deg = np.bincount(g.edges.reshape(-1), minlength=g.n)
+    assert int(deg.max()) > 512 and int((deg >= 256).sum()) >= 8  # hubs, and F above the stage
+    names = ["c4", "diamond", "tailed_triangle", "k4", "house", "c5"]
     ref = {n: O.count(g, T.query(n), "auto", threads=THREADS) for n in names}
-    for min_deg in ("32", "1"):
-        monkeypatch.setenv("TDFS_HASH_MIN_DEG", min_deg)
-        h = M.tdfs_load_edges(g.n, g.edges)
-        for byref in ("1", "0"):  # leaf set F referenced in place vs materialised in shared memory
-            monkeypatch.setenv("TDFS_BYREF", byref)
-            for n in names:
-                p = M.plan_from_query(T.query(n))
-                for fl in (0, M.TDFS_RUN_NO_HUB_BITMAP, M.TDFS_RUN_NO_HASH, M.TDFS_RUN_NO_HASH | M.TDFS_RUN_NO_LEAF_STAGE,
-                           M.TDFS_RUN_NO_HUB_BITMAP | M.TDFS_RUN_NO_LEAF_STAGE | 4):
-                    assert M.tdfs_count(h, p, M.default_opts(flags=fl)) == ref[n], (n, min_deg, byref, fl)
+    words = (g.n + 31) // 32
+    for hub_bytes in (0, -1, 4 * words):
+        h = M.tdfs_load_edges(g.n, g.edges, hub_bitmap_bytes=hub_bytes)
+        for n in names:
+            p = M.plan_from_query(T.query(n))
+            for fl in (0, M.TDFS_RUN_NO_LEAF_STAGE, M.TDFS_RUN_NO_REUSE):
+                assert M.tdfs_count(h, p, M.default_opts(flags=fl)) == ref[n], (n, hub_bytes, fl)
         h.free()
 
 
@@ -251,12 +252,37 @@ def test_order_independence():
 
 
 def test_shard_sum():
+    """Shard-sum invariant for both partitions of the initial edges."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
     rmat12 = graph("r10")
     for name in ["triangle", "diamond", "house"]:
         q = T.query(name)
         ref = oracle_count("r10", q, "auto")
-        for W in (2, 3, 8):
-            assert sum(U.count(rmat12, q, "auto", shard_rank=r, shard_world=W) for r in range(W)) == ref
+        for pol in (M.TDFS_SHARD_ROUND_ROBIN, M.TDFS_SHARD_DEGREE_BALANCED):
+            for W in (2, 3, 8):
+                assert sum(U.count(rmat12, q, "auto", shard_rank=r, shard_world=W, shard_policy=pol)
+                           for r in range(W)) == ref, (name, pol, W)
+
+
+def test_degree_balanced_shards_match_oracle_on_owned_edges():
+    """A degree-balanced shard counts exactly the matches whose root edge it owns: the oracle
+    restricted to one round-robin shard of W' = nnz (a single edge) summed over the edges
+    tdfs_partition_edges gives rank r equals the kernel's rank-r count (small graph)."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    g = T.rmat(8, 6, 5)
+    offs, adj = T.to_csr(g)
+    W = 3
+    own = M.tdfs_partition_edges(offs, adj, W, M.TDFS_SHARD_DEGREE_BALANCED)
+    q = T.query("diamond")
+    order = O.oracle_order(q)
+    nnz = adj.shape[0]
+    og = O.OracleGraph(g)
+    per_edge = [O.count(og, q, "auto", order=order, shard=(e, nnz)) for e in range(nnz)]
+    for r in range(W):
+        want = sum(c for c, o in zip(per_edge, own) if o == r)
+        got = U.count(g, q, "auto", order=order, shard_rank=r, shard_world=W,
+                      shard_policy=M.TDFS_SHARD_DEGREE_BALANCED)
+        assert got == want, r
 
 
 def test_labeled_queries():
@@ -393,9 +419,17 @@ def test_config2_full_sampled_shards(c2, name):
         assert got == ref, (name, r)
 
 
-def test_config2_auto_order_full_counts_equal_explicit_order(c2):
-    """The planner's own order (what bench.py runs) gives the same full count as the
-    oracle-order run whose shards are checked above."""
-    for name in ["c4", "diamond", "tailed_triangle", "k4"]:
+def test_config2_full_counts_equal_oracle_goldens(c2):
+    """The five benched C2 counts, in bench.py's launch configuration (planner order, tau = 10 ms,
+    chunk 8 / 1), equal the oracle's full-graph counts, written to tests/golden/c2_counts.txt by
+    scripts/golden_counts.py (oracle/ only; M is order-independent, R9)."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    gold = {k: int(v.split()[0]) for k, v in G.read("c2_counts.txt").items()}
+    assert set(gold) >= set(T.CONFIG_QUERIES[2])
+    h = U.load(c2)
+    for name in T.CONFIG_QUERIES[2]:
         q = T.query(name)
-        assert U.count(c2, q, "auto") == U.count(c2, q, "auto", order=O.oracle_order(q))
+        o = M.default_opts(chunk=8 if q.k <= 3 else 1)
+        assert M.tdfs_count(h, M.plan_from_query(q), o) == gold[name], name
+        if name != "triangle":  # and the oracle-order plan whose shards are checked above
+            assert U.count(c2, q, "auto", order=O.oracle_order(q)) == gold[name], name

@@ -269,8 +269,9 @@ def test_nodes_and_W_triangle_closed_form():
 
 
 def test_W_stream_triangle_closed_form():
-    """R29b roofline bytes for the triangle, order [0,1,2], constraints 0<1<2: each internal
-    prefix (edge u<v, both degrees >= 2) adds 2 x 16 B + 4 B x min(|N(u) > v|, |N(v) > v|)."""
+    """R32 roofline bytes for the triangle, order [0,1,2], constraints 0<1<2: each internal
+    prefix (edge u<v, both degrees >= 2) adds 2 x 16 B + 4 B x min(|N(u) > v|, |N(v) > v|)
+    (no earlier candidate set can be a source at position 2)."""
     g = T.rmat(10, 8, 13)
     d = _degrees(g)
     nbrs = [[] for _ in range(g.n)]
@@ -285,6 +286,29 @@ def test_W_stream_triangle_closed_form():
     # a count-only single-operand last position streams nothing: wedge = 16 B per prefix
     r = O.match(g, T.query("wedge"), "auto", order=[0, 1, 2])
     assert r["W_stream"] == 16 * r["nodes"][1]
+
+
+def test_W_stream_diamond_reuse_closed_form():
+    """R32 with a reuse source: diamond in the planner's order [1, 2, 0, 3]
+    with C_auto = {u0 < u3, u1 < u2}.  Position 2 (u0, B = {p0, p1}, no window) adds
+    32 B + 4 B x min(deg a, deg b) per edge prefix a < b with deg >= 3; position 3 (u3, same
+    B, window > S[2]) has C(2) as a source that alone is its candidate set, so it is count-only:
+    32 B per prefix (a, b, c), c any common neighbour.  Closed form with numpy (A @ A)."""
+    g = T.rmat(9, 8, 17)
+    n = g.n
+    A = np.zeros((n, n), dtype=np.int64)
+    A[g.edges[:, 0], g.edges[:, 1]] = 1
+    A[g.edges[:, 1], g.edges[:, 0]] = 1
+    d = A.sum(1)
+    common = A @ A
+    tot = 0
+    for a, b in g.edges.tolist():  # a < b (canonical), the edge constraint S0 < S1
+        if d[a] >= 3 and d[b] >= 3:
+            tot += 32 + 4 * int(min(d[a], d[b])) + 32 * int(common[a, b])
+    q = T.query("diamond")
+    assert O.automorphisms(q)[1] == [(0, 3), (1, 2)]
+    r = O.match(g, q, "auto", order=[1, 2, 0, 3])
+    assert r["W_stream"] == tot
 
 
 def test_enumerate_tuples_satisfy_definition():
