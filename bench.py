@@ -446,6 +446,8 @@ def run_ours(a):
                                  "timeouts": int(stats_runs[i]["timeouts"]),
                                  "tasks_enqueued": int(stats_runs[i]["tasks_enqueued"]),
                                  "pages_used": int(stats_runs[i]["pages_used"]),
+                                 "warp_exit_ms_first_mean_last_stats_run": [
+                                     round(stats_runs[i][f"warp_exit_{x}_ns"] / 1e6, 3) for x in ("first", "mean", "last")],
                                  "nodes_per_level": stats_runs[i]["nodes_per_level"][:q.k]}
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,

@@ -195,9 +195,13 @@ typedef struct {
   float kernel_ms;            /* CUDA-event time of the matching kernel */
   int32_t grid_blocks, warps_per_block, page_table_entries, pad_;
   uint64_t pool_pages;
-  uint64_t stream_bytes;      /* roofline bytes (R29b): sum over extensions of 16 B per Eq. (1)
-                                 operand + 4 B x |smallest constraint-windowed operand| (0 for a count-only
-                                 last position with one operand and no label test) */
+  uint64_t stream_bytes;      /* roofline bytes (R32): sum over extensions of 16 B per Eq. (1)
+                                 operand + 4 B x |smallest constraint-windowed Eq. (1) source| (operands and
+                                 reusable earlier candidate sets; 0 for a count-only last position) */
+  uint64_t warp_exit_first_ns; /* load balance inside the GPU: when the first / an average / the last warp */
+  uint64_t warp_exit_mean_ns;  /*   last found no work (queue empty, edges exhausted), from the kernel's first */
+  uint64_t warp_exit_last_ns;  /*   warp start (ns); last - mean is the straggler tail that timeout
+                                  splitting shortens */
 } tdfs_stats;
 
 /* Bytes of caller-owned device workspace needed for one job (256-byte aligned). */
@@ -222,6 +226,24 @@ int tdfs_count(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, 
 int tdfs_enumerate(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, void* workspace,
                    size_t ws_bytes, void* stream, int32_t* d_out, uint64_t cap, uint64_t* n_total,
                    tdfs_stats* stats);
+
+/* Streaming enumerate ("output S"): every match of this shard,
+ * without a capacity limit.  The kernel writes tuples (indexed by query vertex id, as in
+ * tdfs_enumerate) into the caller-owned device ring d_ring[ring_cap * k] and waits for free space;
+ * the calling thread drains it chunk by chunk (ring_cap / 8 tuples, copied to pinned host memory on
+ * a side stream while the kernel runs) into sink(tuples, n, k, user) -- host memory valid during the
+ * call only; a nonzero return stops delivery (the kernel still finishes and *n_total stays exact;
+ * the call then returns TDFS_E_INVALID_ARG).  Synchronous.  ring_cap: positive multiple of 8.
+ * Errors: as tdfs_count, plus INVALID_ARG. */
+typedef int (*tdfs_tuple_sink)(const int32_t* tuples, uint64_t n, int32_t k, void* user);
+int tdfs_enumerate_stream(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, void* workspace,
+                          size_t ws_bytes, void* stream, int32_t* d_ring, uint64_t ring_cap, tdfs_tuple_sink sink,
+                          void* user, uint64_t* n_total);
+/* tdfs_enumerate_stream into a rank-local binary file: n_total rows of k little-endian int32
+ * (query-vertex order), no header; tuples in no particular order. */
+int tdfs_enumerate_to_file(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, void* workspace,
+                           size_t ws_bytes, void* stream, int32_t* d_ring, uint64_t ring_cap, const char* path,
+                           uint64_t* n_total);
 
 /* Status of the last job run in `workspace` (device-side error word), synchronising `stream`. */
 int tdfs_workspace_status(const void* workspace, void* stream);

@@ -86,7 +86,9 @@ class tdfs_stats(ctypes.Structure):
                 ("edges_scanned", ctypes.c_uint64), ("edges_filtered_in", ctypes.c_uint64),
                 ("chunks_fetched", ctypes.c_uint64), ("kernel_ms", ctypes.c_float), ("grid_blocks", ctypes.c_int32),
                 ("warps_per_block", ctypes.c_int32), ("page_table_entries", ctypes.c_int32), ("pad_", ctypes.c_int32),
-                ("pool_pages", ctypes.c_uint64), ("stream_bytes", ctypes.c_uint64)]
+                ("pool_pages", ctypes.c_uint64), ("stream_bytes", ctypes.c_uint64),
+                ("warp_exit_first_ns", ctypes.c_uint64), ("warp_exit_mean_ns", ctypes.c_uint64),
+                ("warp_exit_last_ns", ctypes.c_uint64)]
 
     def as_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f not in ("nodes_per_level", "pad_")}
@@ -124,6 +126,10 @@ SIGNATURES = {
     "tdfs_enumerate": (ctypes.c_int, [_vp, _vp, ctypes.POINTER(tdfs_run_opts), _vp, ctypes.c_size_t, _vp, _vp,
                                       ctypes.c_uint64, _u64p, ctypes.POINTER(tdfs_stats)]),
     "tdfs_workspace_status": (ctypes.c_int, [_vp, _vp]),
+    "tdfs_enumerate_stream": (ctypes.c_int, [_vp, _vp, ctypes.POINTER(tdfs_run_opts), _vp, ctypes.c_size_t, _vp, _vp,
+                                             ctypes.c_uint64, _vp, _vp, _u64p]),
+    "tdfs_enumerate_to_file": (ctypes.c_int, [_vp, _vp, ctypes.POINTER(tdfs_run_opts), _vp, ctypes.c_size_t, _vp,
+                                              _vp, ctypes.c_uint64, ctypes.c_char_p, _u64p]),
     "tdfs_partition_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, ctypes.c_int32, ctypes.c_int32,
                                             _vp]),
     "tdfs_shared_cursor_create": (ctypes.c_int, [ctypes.c_int, ctypes.POINTER(_vp), _vp]),
@@ -402,53 +408,119 @@ def tdfs_enumerate(g: GraphHandle, p: PlanHandle, cap: int, opts: Optional[tdfs_
 
 def tdfs_enumerate_chunks(g: GraphHandle, p: PlanHandle, chunk_cap: int, opts: Optional[tdfs_run_opts] = None,
                           workspace=None, stream=None):
-    """Enumerate every match in chunks of at most `chunk_cap` tuples, streamed to pinned host
-    memory ("output S").
+    """Enumerate every match of this caller's shard as a generator of (tuples, total_so_far), tuples
+    an (n <= chunk_cap, k) int32 numpy array indexed by query vertex id.
 
-    Marshalling only -- all matching runs in tdfs_count / tdfs_enumerate.  The initial edge
-    tasks of this caller's shard (opts.shard_rank / shard_world; a multi-GPU rank streams its
-    rank-local output) are refined into round-robin sub-shards (r + W*s of W*S),
-    S sized from one count pass so that each sub-shard's tuples fit one device buffer of
-    chunk_cap * k ints; a sub-shard that still overflows is split in two.  Yields
-    (tuples (n, k) int32 numpy array, total_so_far); tuples are indexed by query vertex id."""
-    torch = _torch()
-    opts = opts or default_opts()
+    Marshalling only: one tdfs_enumerate_stream job (the kernel writes into a device ring of
+    8 * ceil(chunk_cap / 8) tuples drained by the library) runs on a helper thread; its sink hands
+    each drained chunk to this generator through a bounded queue, so a slow consumer back-pressures
+    the kernel (its warps wait for ring space) instead of buffering without bound."""
+    import queue
+    import threading
+
     if chunk_cap < 1:
         raise TdfsError(TDFS_E_INVALID_ARG, "chunk_cap must be >= 1")
-    k = p.k
-    base_r, base_w = int(opts.shard_rank), int(opts.shard_world)
-    total = tdfs_count(g, p, opts, workspace=workspace, stream=stream)
-    if total == 0:
-        return
-    out = torch.empty(chunk_cap * k, dtype=torch.int32, device=f"cuda:{g.device}")
-    host = torch.empty(chunk_cap * k, dtype=torch.int32, pin_memory=True)
-    # ~2x headroom for uneven sub-shards, capped (a sub-shard that overflows is split again)
-    S = min(max(1, -(-2 * total // chunk_cap)), 4096)
-    todo = [(base_r + base_w * s, base_w * S) for s in range(S - 1, -1, -1)]
+    ring_cap = 8 * max(1, -(-chunk_cap // 8))
+    q: "queue.Queue" = queue.Queue(maxsize=2)
+    stop = threading.Event()
+    res = {}
+
+    def sink(arr):
+        for i in range(0, arr.shape[0], chunk_cap):
+            while True:
+                if stop.is_set():
+                    return True
+                try:
+                    q.put(arr[i:i + chunk_cap], timeout=0.1)
+                    break
+                except queue.Full:
+                    continue
+        return False
+
+    def run():
+        try:
+            res["total"] = tdfs_enumerate_stream(g, p, sink, ring_cap, opts, workspace, stream)
+        except BaseException as e:  # noqa: BLE001 -- re-raised in the generator
+            res["error"] = e
+        finally:
+            q.put(None)
+
+    th = threading.Thread(target=run, daemon=True)
+    th.start()
     done = 0
-    while todo:
-        r, w = todo.pop()
-        if w >= 2**31 - 1:
-            raise TdfsError(TDFS_E_INVALID_ARG, "a single initial edge has more than chunk_cap matches")
-        o = tdfs_run_opts.from_buffer_copy(opts)
-        o.shard_rank, o.shard_world = r, w
-        tot = ctypes.c_uint64(0)
-        nbytes = tdfs_workspace_bytes(g, p, o)
-        ws = _ws_for(g, nbytes, workspace)
-        rc = _lib.tdfs_enumerate(g.ptr, p.ptr, ctypes.byref(o), ws.data_ptr(), ws.numel(), _stream_ptr(stream, g.device),
-                                 out.data_ptr(), int(chunk_cap), ctypes.byref(tot), None)
-        _check(rc, allow=(TDFS_E_OUTPUT_OVERFLOW,))
-        if rc == TDFS_E_OUTPUT_OVERFLOW:  # split this sub-shard in two: r and r + w of 2w
-            todo += [(r + w, 2 * w), (r, 2 * w)]
-            continue
-        n = int(tot.value)
-        if n == 0:
-            continue
-        host[: n * k].copy_(out[: n * k])
-        done += n
-        yield host[: n * k].view(n, k).numpy().copy(), done
-    if done != total:
-        raise TdfsError(TDFS_E_CUDA, f"chunked enumeration produced {done} tuples, count pass {total}")
+    try:
+        while True:
+            item = q.get()
+            if item is None:
+                break
+            done += item.shape[0]
+            yield item, done
+    finally:
+        stop.set()
+        while th.is_alive():
+            try:
+                q.get(timeout=0.1)
+            except queue.Empty:
+                pass
+        th.join()
+    if "error" in res:
+        raise res["error"]
+    if res.get("total") != done:
+        raise TdfsError(TDFS_E_CUDA, f"streamed {done} tuples, job total {res.get('total')}")
+
+
+TUPLE_SINK = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(ctypes.c_int32), ctypes.c_uint64, ctypes.c_int32,
+                              ctypes.c_void_p)
+
+
+def _ring(g: GraphHandle, k: int, ring_cap: int):
+    torch = _torch()
+    if ring_cap < 8 or ring_cap % 8:
+        raise TdfsError(TDFS_E_INVALID_ARG, "ring_cap must be a positive multiple of 8")
+    return torch.empty(ring_cap * k, dtype=torch.int32, device=f"cuda:{g.device}")
+
+
+def tdfs_enumerate_stream(g: GraphHandle, p: PlanHandle, sink, ring_cap: int = 1 << 20,
+                          opts: Optional[tdfs_run_opts] = None, workspace=None, stream=None) -> int:
+    """Stream every match (NEXT-2): sink(tuples) receives (n, k) int32 numpy arrays (a copy), indexed
+    by query vertex id; returning True stops delivery.  Returns the exact total."""
+    opts = opts or default_opts()
+    k = p.k
+    ring = _ring(g, k, ring_cap)
+    ws = _ws_for(g, tdfs_workspace_bytes(g, p, opts), workspace)
+    err = []
+
+    def _cb(ptr, n, kk, user):
+        try:
+            arr = np.ctypeslib.as_array(ptr, shape=(int(n) * int(kk),)).reshape(int(n), int(kk)).copy()
+            return 1 if sink(arr) else 0
+        except Exception as e:  # noqa: BLE001 -- re-raised after the call
+            err.append(e)
+            return 1
+
+    cb = TUPLE_SINK(_cb)
+    tot = ctypes.c_uint64(0)
+    rc = _lib.tdfs_enumerate_stream(g.ptr, p.ptr, ctypes.byref(opts), ws.data_ptr(), ws.numel(),
+                                    _stream_ptr(stream, g.device), ring.data_ptr(), int(ring_cap),
+                                    ctypes.cast(cb, ctypes.c_void_p), None, ctypes.byref(tot))
+    if err:
+        raise err[0]
+    _check(rc)
+    return int(tot.value)
+
+
+def tdfs_enumerate_to_file(g: GraphHandle, p: PlanHandle, path: str, ring_cap: int = 1 << 20,
+                           opts: Optional[tdfs_run_opts] = None, workspace=None, stream=None) -> int:
+    """Every match of this shard (opts.shard_rank / shard_world: a rank-local file) into `path`:
+    raw int32 rows of k ids (query-vertex order).  Returns the exact total."""
+    opts = opts or default_opts()
+    ring = _ring(g, p.k, ring_cap)
+    ws = _ws_for(g, tdfs_workspace_bytes(g, p, opts), workspace)
+    tot = ctypes.c_uint64(0)
+    _check(_lib.tdfs_enumerate_to_file(g.ptr, p.ptr, ctypes.byref(opts), ws.data_ptr(), ws.numel(),
+                                       _stream_ptr(stream, g.device), ring.data_ptr(), int(ring_cap),
+                                       os.fsencode(path), ctypes.byref(tot)))
+    return int(tot.value)
 
 
 def tdfs_workspace_status(workspace, stream=None, device: int = 0) -> int:

@@ -2,6 +2,7 @@
 // defaults, workspace sizing and the count / enumerate entry points (tdfs.h).
 #include <cuda_runtime.h>
 
+#include <cstdio>
 #include <cstring>
 #include <string>
 
@@ -94,6 +95,45 @@ extern "C" int tdfs_enumerate(const tdfs_graph* g, const tdfs_plan* p, const tdf
   }
   return launch_job(graph_of(g), plan_of(p), o, workspace, ws_bytes, stream, 1, d_out, cap, nullptr, true, n_total,
                     stats, nullptr, 0, nullptr);
+}
+
+extern "C" int tdfs_enumerate_stream(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, void* workspace,
+                                     size_t ws_bytes, void* stream, int32_t* d_ring, uint64_t ring_cap,
+                                     tdfs_tuple_sink sink, void* user, uint64_t* n_total) {
+  if (!g || !p) return fail(TDFS_E_INVALID_ARG, "enumerate_stream: NULL graph or plan");
+  tdfs_run_opts d;
+  if (!o) {
+    tdfs_run_opts_default(&d);
+    o = &d;
+  }
+  return stream_job(graph_of(g), plan_of(p), o, workspace, ws_bytes, stream, d_ring, ring_cap, sink, user, n_total);
+}
+
+namespace {
+struct FileSink {
+  FILE* f;
+  bool bad;
+};
+int file_sink(const int32_t* t, uint64_t n, int32_t k, void* user) {
+  FileSink* s = static_cast<FileSink*>(user);
+  if (std::fwrite(t, sizeof(int32_t) * (size_t)k, (size_t)n, s->f) != (size_t)n) {
+    s->bad = true;
+    return 1;
+  }
+  return 0;
+}
+}  // namespace
+
+extern "C" int tdfs_enumerate_to_file(const tdfs_graph* g, const tdfs_plan* p, const tdfs_run_opts* o, void* workspace,
+                                      size_t ws_bytes, void* stream, int32_t* d_ring, uint64_t ring_cap,
+                                      const char* path, uint64_t* n_total) {
+  if (!path) return fail(TDFS_E_INVALID_ARG, "enumerate_to_file: NULL path");
+  FileSink s{std::fopen(path, "wb"), false};
+  if (!s.f) return fail(TDFS_E_INVALID_ARG, std::string("enumerate_to_file: cannot open ") + path);
+  int rc = tdfs_enumerate_stream(g, p, o, workspace, ws_bytes, stream, d_ring, ring_cap, file_sink, &s, n_total);
+  if (std::fclose(s.f) != 0 && rc == TDFS_OK) rc = fail(TDFS_E_INVALID_ARG, "enumerate_to_file: write failed");
+  if (s.bad) rc = fail(TDFS_E_INVALID_ARG, std::string("enumerate_to_file: write failed: ") + path);
+  return rc;
 }
 
 extern "C" int tdfs_workspace_status(const void* workspace, void* stream) {

@@ -29,7 +29,10 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
 constexpr int kBlockThreads = 128;  // matching-kernel block size (its __launch_bounds__)
-constexpr int kLeafStage = 512;  // default shared-memory ids per warp for the leaf set F
+#ifndef TDFS_LEAF_STAGE
+#define TDFS_LEAF_STAGE 512
+#endif
+constexpr int kLeafStage = TDFS_LEAF_STAGE;  // shared-memory ids per warp for the leaf set F
 // Hub bitmaps (graph.cu): vertices of degree >= kHubMinDeg, highest first, within the budget
 constexpr int64_t kHubMinDeg = 256;
 constexpr int64_t kHubBudgetDefault = 256ll << 20;
@@ -94,15 +97,23 @@ struct Graph {
 };
 
 // ---------------------------------------------------------------- device job
-struct QSlot {                // one task of Q_task, 32 bytes (one sector; PAPER.md:191 uses 3 ints)
-  int32_t v1, v2, v3;         // <v1,v2,-2> edge task, <v1,v2,v3> 3-prefix task
-  int32_t v4;                 // -1, or the id range end of a range task <v1,v2,lo,hi>
+// One task of Q_task, 32 bytes (one sector; PAPER.md:191 uses 3 ints).  hdr = kind | level << 4:
+//   TASK_EDGE    <v1, v2>              an initial edge task (PAPER.md:189 <v1,v2,-2>), DFS from level 2
+//   TASK_PREFIX  <v1, v2, v3>          a 3-prefix task, DFS from level 3
+//   TASK_RANGE   <S0 .. S_{d-1}, lo, hi>  level d (2 <= d <= 4) candidates of that prefix with ids in
+//                                      [lo, hi) (R30/R33 range tasks), DFS from level d
+constexpr int TASK_EDGE = 0, TASK_PREFIX = 1, TASK_RANGE = 2;
+constexpr int kMaxRangeLevel = 4;  // d + 2 ints (prefix, lo, hi) fit the 6 payload words
+struct QSlot {
+  int32_t hdr;
+  int32_t v[6];
   uint32_t seq;               // ticket handshake: == t free for ticket t, == t+1 full for ticket t
-  uint32_t pad[3];
 };
+static_assert(sizeof(QSlot) == 32, "one 32-byte sector per task");
 
 enum CounterIdx {            // each counter on its own 128-byte line
   C_COUNT = 0, C_CURSOR, C_QHEAD, C_QTAIL, C_QAVAIL, C_QFREE, C_ACTIVE, C_POOL, C_ERROR, C_OUTCUR, C_TRACE,
+  C_CONSUMED,                  // streaming enumerate: tuples the host has drained (written by the host)
   C_NUM
 };
 constexpr int kCounterStride = 16;  // u64 words per counter (128 B)
@@ -110,6 +121,8 @@ constexpr int kCounterStride = 16;  // u64 words per counter (128 B)
 enum StatIdx {
   S_NODES = 0,                 // 9 entries
   S_ADJ_BYTES = 9, S_ENQ, S_DEQ, S_TIMEOUTS, S_QFULL, S_EDGES_SCANNED, S_EDGES_IN, S_CHUNKS, S_STREAM,
+  S_T_START,                   // min over warps of the start time (%globaltimer ns)
+  S_T_EXIT_MIN, S_T_EXIT_MAX, S_T_EXIT_SUM, S_WARPS,  // warp exit times (absolute ns; sum over warps)
   S_NUM
 };
 
@@ -144,9 +157,11 @@ struct KParams {
   int64_t tau_ns;              // < 0: infinity
   int32_t fcap;                // leaf staging: shared-memory ids per warp (0 = off)
   int32_t meta_off;            // shared-memory layout: byte offset of the warps' leaf-batch entries
-  int32_t range_split;         // k = 4: split level 2 into <= 32 id-range tasks (else one task per sibling, R30)
-  int32_t range_ok;            // the plan uses range tasks (see launch_job)
-  int32_t reuse2_used;         // a later position / the leaf set reuses position 2's list (range tasks build it whole)
+  uint32_t split_mask;         // bit d: level d is split-eligible -- 2 (the paper's rule) and the
+                               // range-task levels up to kMaxRangeLevel (R33)
+  uint32_t range_mask;         // bit d: a timed-out level d splits into <= 32 id-range tasks (R30/R33); level 2
+                               // without the bit pushes one <S0,S1,v> task per sibling
+  uint32_t reused_mask;        // bit d: a later position / the leaf set reuses C(d) (range tasks then build it whole)
   // initial edge tasks: j -> directed edge task_edges[j] (shard list) or shard_rank + j * shard_world
   const int32_t* task_edges;   // nullptr = arithmetic shard
   unsigned long long* gcursor; // chunk cursor: this job's counter, or a cross-rank shared one (NEXT-3)
@@ -158,14 +173,18 @@ struct KParams {
   // enumerate
   int32_t* out;
   unsigned long long cap;
+  unsigned long long ring_chunk;   // streaming (NEXT-2): tuples per ring chunk, 0 = capacity mode
+  unsigned long long ring_nchunks;
+  unsigned long long* ring_fill;   // [ring_nchunks] tuples written into each chunk (reset by the host)
   // tracing (tests)
   int32_t* trace;
   long long trace_cap;
 };
 
 // workspace layout (byte offsets from the 256-aligned base)
+constexpr int kRingChunks = 8;  // streaming enumerate: the output ring is drained in 8 chunks
 struct WsLayout {
-  size_t ctr = 0, stats = 0, slots = 0, tables = 0, pool = 0, total = 0;
+  size_t ctr = 0, stats = 0, fill = 0, slots = 0, tables = 0, pool = 0, total = 0;
   uint64_t qcap = 0, qslots = 0, n_pages = 0;
   int32_t E = 0, page_shift = 0, n_levels = 0, blocks = 0, wpb = 0, fcap = 0;
 };
@@ -174,7 +193,11 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
 int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
                int mode /*0 count, 1 enumerate*/, int32_t* d_out, uint64_t cap, uint64_t* d_count,
                bool sync, uint64_t* h_count, tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap,
-               int64_t* n_trace);
+               int64_t* n_trace, bool ring = false);
+// streaming enumerate (match.cu): launch in ring mode, then drain chunks to sink until the job ends
+typedef int (*SinkFn)(const int32_t* tuples, uint64_t n, int32_t k, void* user);
+int stream_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
+               int32_t* d_ring, uint64_t ring_cap, SinkFn sink, void* user, uint64_t* n_total);
 int blocks_per_sm(int device, int wpb, bool stats, bool enumerate, int fcap, int* out);
 const Graph* graph_of(const tdfs_graph* g);
 // host partition of the directed edges (tdfs_partition_edges) and the device task list of one rank

@@ -32,7 +32,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <climits>
+#include <thread>
 #include <cstdlib>
 #include <cstring>
 
@@ -53,8 +55,11 @@ struct __align__(16) LeafMeta {
   int s, e;      // streamed element range: stream A F-coordinates [s, e) of the 16-byte aligned F,
                  // stream B N(x) entries [b0 + s, b0 + e) (narrowed to [F_min, F_max])
 };
-// 32 entries + 33 prefix ints, padded to 16 B
-constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144;
+// 32 entries + 33 prefix ints (padded to 16 B) + a 128-id transpose buffer
+#ifndef TDFS_TRANSPOSE
+#define TDFS_TRANSPOSE 1
+#endif
+constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144 + (TDFS_TRANSPOSE ? 512 : 0);
 __host__ __device__ inline size_t smem_meta_offset(int wpb, int fcap) {
   return ((size_t)wpb * fcap * sizeof(int) + 15) & ~(size_t)15;
 }
@@ -76,9 +81,13 @@ struct Ctx {
   unsigned long long wbytes, sbytes, enq, deq, touts, qfull, scanned, edges_in, chunks;  // lane 0 (STATS)
   uint32_t* tables;         // this warp's page tables [n_levels][E]
   int* sF;                  // this warp's shared-memory stage for the leaf set F (P.fcap ints)
-  int w2lo, w2hi;           // range task: its level-2 candidates are the ids in [w2lo, w2hi) (warp-uniform)
-  int w2mode;               // 0 no range task; 1 level 2 built as the slice only; 2 built whole, iterated in the slice
-  int end2;                 // mode 2: iteration end index of level 2 (INT_MAX otherwise)
+  int wlev;                 // range task: level d whose candidates are restricted to ids in [wlo, whi); 0 = none
+  int wlo, whi;
+  int wmode;                // 1: level wlev built as the slice only; 2: built whole, iterated in the slice
+  int wend;                 // mode 2: iteration end index at level wlev (INT_MAX otherwise)
+  int own;                  // lowest stored level whose FULL candidate list this warp built for the current
+                            // prefix (2 for edge tasks, 3 for 3-prefix tasks, wlev / wlev+1 for range tasks):
+                            // only lists at levels >= own may be reused (set-intersection reuse)
 };
 
 __device__ __forceinline__ int getS(int sreg, int p) { return __shfl_sync(FULL, sreg, p); }
@@ -137,6 +146,26 @@ __device__ __forceinline__ long long warp_paged_lower_bound(const KParams& P, co
   return lo + __popc(__ballot_sync(FULL, less));
 }
 
+// Enumerate output of match number idx, t[p] = f(pi_p) (written indexed by query vertex id).
+// Capacity mode (P.ring_chunk == 0): out[idx] if idx < cap, else dropped (the total stays exact).
+// Streaming mode (NEXT-2): out is a ring of cap tuples in ring_chunk-tuple chunks drained by the
+// host (tdfs_enumerate_stream); the lane waits until its slot is free (idx < consumed + cap), writes
+// the tuple, and counts it into its chunk's fill word; the host copies a chunk out once it is full.
+// A lane only waits for its own slot, so the chunk the host waits for always completes.
+__device__ __forceinline__ void emit_tuple(const KParams& P, unsigned long long idx, const int* t, int k) {
+  if (P.ring_chunk == 0) {
+    if (idx < P.cap)
+      for (int p = 0; p < k; p++) P.out[idx * k + P.plan.order[p]] = t[p];
+    return;
+  }
+  const unsigned long long* consumed = ctr(P, C_CONSUMED);
+  while (idx >= (unsigned long long)ld_relaxed_s64(consumed) + P.cap) __nanosleep(2000);
+  const unsigned long long slot = idx % P.cap;
+  for (int p = 0; p < k; p++) P.out[slot * k + P.plan.order[p]] = t[p];
+  __threadfence();
+  atomicAdd(P.ring_fill + (idx / P.ring_chunk) % P.ring_nchunks, 1ull);
+}
+
 // STATS only (roofline bytes R32): |C(r) within [lo, hi)| from the definition, for a stored
 // position r whose list this warp did not build (a <v1,v2,v3> or range task): the ids of the
 // intersection of r's backward lists inside r's window and [lo, hi) that pass r's injectivity,
@@ -182,15 +211,14 @@ __device__ long long source_size_def(const KParams& P, Ctx<STATS>& c, int r, int
 //           2 = enumerate (last position); 3 = stage into shared memory (d = kVF, the
 //           S[k-2]-independent part of the last position), or return -2 without
 //           writing when the streamed operand exceeds the stage (P.fcap ids).
-// allow_reuse2: the stored list of position 2 belongs to this prefix (false for tasks
-// <v1,v2,v3> taken from Q_task, whose level 2 was built by another warp).
+// Set-intersection reuse starts only from lists this warp built in full (levels >= c.own).
 // Returns the number of candidates, or -1 on stack exhaustion.
 template <int MODE_OUT, bool STATS>
-__device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_reuse2) {
+__device__ long long extend(const KParams& P, Ctx<STATS>& c, int d) {
   const int lane = c.lane;
   const DevPlan& pl = P.plan;
   int r = pl.reuse[d];
-  if (r == 2 && !allow_reuse2) r = -1;
+  if (r >= 0 && r < c.own) r = -1;
   const uint32_t bm_all = pl.bwd[d];
   // set-intersection result reuse: start from C(r), intersect the rest
   const uint32_t bm = (r >= 0) ? (bm_all & ~pl.bwd[r]) : bm_all;
@@ -211,7 +239,7 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
     if (P.hub_id) hid = __ldg(P.hub_id + sj);
   }
   // a range task re-extends part of a level-2 list its splitter already counted (STATS only)
-  const bool counted = STATS && MODE_OUT != 3 && !(d == 2 && c.w2mode != 0);
+  const bool counted = STATS && MODE_OUT != 3 && d != c.wlev;
   if (counted) {  // W of SURVEY 8(d) counts every backward operand of Eq. (1), reused or not
     const bool mine = (bm_all >> lane) & 1u;
     unsigned long long wb = 0;
@@ -223,9 +251,9 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
   const uint32_t lom = pl.lo_mask[d], him = pl.hi_mask[d];
   int lo = __reduce_max_sync(FULL, (lom >> lane & 1u) ? c.sreg + 1 : 0);
   int hi = (int)__reduce_min_sync(FULL, (him >> lane & 1u) ? (unsigned)c.sreg : (unsigned)INT_MAX);
-  if (d == 2 && c.w2mode == 1) {  // range task: only the level-2 candidates in [w2lo, w2hi)
-    lo = max(lo, c.w2lo);
-    hi = min(hi, c.w2hi);
+  if (d == c.wlev && c.wmode == 1) {  // range task: only the level-d candidates in [wlo, whi)
+    lo = max(lo, c.wlo);
+    hi = min(hi, c.whi);
   }
   if (counted) {  // roofline bytes R32: 16 B per operand + 4 B x the smallest windowed Eq. (1) source
     const bool mine = (bm_all >> lane) & 1u;
@@ -242,8 +270,8 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       for (uint32_t sm = pl.src_mask[d]; sm; sm &= sm - 1) {  // stored candidate sets C(r) (reuse sources)
         const int rr = __ffs(sm) - 1;
         long long len;
-        if (rr == 2 && !allow_reuse2) {
-          len = source_size_def(P, c, rr, lo, hi);  // level 2 not built by this warp: from the definition
+        if (rr < c.own) {
+          len = source_size_def(P, c, rr, lo, hi);  // list not built (in full) by this warp: from the definition
         } else {
           const uint32_t* tb = c.tables + (size_t)(rr - 2) * P.E;
           const long long rs = __shfl_sync(FULL, c.lsize, rr);
@@ -412,11 +440,11 @@ __device__ long long extend(const KParams& P, Ctx<STATS>& c, int d, bool allow_r
       ob0 = __shfl_sync(FULL, ob0, 0);
       const int k = pl.k;
       const unsigned long long idx = ob0 + __popc(bal & lanemask_lt());
-      for (int p = 0; p < k - 1; p++) {
-        const int s = getS(c.sreg, p);
-        if (ok && idx < P.cap) P.out[idx * k + pl.order[p]] = s;
-      }
-      if (ok && idx < P.cap) P.out[idx * k + pl.order[k - 1]] = v;
+      int t[kMaxK];
+#pragma unroll
+      for (int p = 0; p < kMaxK - 1; p++) t[p] = getS(c.sreg, p);
+      t[k - 1] = v;
+      if (ok) emit_tuple(P, idx, t, k);
     }
     total += cnt;
   }
@@ -570,6 +598,11 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
   char* const wbase = reinterpret_cast<char*>(tdfs_smem) + P.meta_off + (int)(threadIdx.x >> 5) * kMetaBytesPerWarp;
   LeafMeta* meta = reinterpret_cast<LeafMeta*>(wbase);
   int* pre = reinterpret_cast<int*>(wbase + 32 * sizeof(LeafMeta));
+  // 128-id transpose buffer: a lane loads 4 consecutive ids with one 128-bit load, but the probes
+  // of ids 4L..4L+3 by lane L would hit 4 sectors per lane; after the transpose lane L probes ids
+  // L, L+32, L+64, L+96 of the warp's 128, so adjacent lanes probe adjacent sorted ids (shared
+  // bitmap words / sectors) -- measured 17.9 sectors per warp load request before
+  int* const tb = reinterpret_cast<int*>(wbase + 32 * sizeof(LeafMeta) + 144);
   if (act) {
     LeafMeta e;
     e.b0 = m.b0;
@@ -594,6 +627,8 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     long long b0j = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
+      int4 q = make_int4(-1, -1, -1, -1);
+      bool k0 = false, k1 = false, k2 = false, k3 = false;
       if (idx < tot) {
         if (idx >= jn) {  // move to the leaf holding idx (per lane, shared-memory reads)
           do { ++j; jn = pre[j + 1]; } while (jn <= idx);
@@ -605,15 +640,33 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
           g0 = sj >> 2;
         }
         const int g = g0 + idx - pj;
-        const int4 q = *reinterpret_cast<const int4*>(Fal + 4 * g);
+        q = *reinterpret_cast<const int4*>(Fal + 4 * g);
         const int i0 = 4 * g;
-        const bool k0 = i0 >= sj && i0 < ej, k1 = i0 + 1 >= sj && i0 + 1 < ej;
-        const bool k2 = i0 + 2 >= sj && i0 + 2 < ej, k3 = i0 + 3 >= sj && i0 + 3 < ej;
-        if (hidj >= 0) {
-          const uint32_t* row = P.hub_bits + (long long)hidj * P.hub_words;
-          cnt += (k0 ? bit_of(row, q.x) : 0u) + (k1 ? bit_of(row, q.y) : 0u) + (k2 ? bit_of(row, q.z) : 0u) +
-                 (k3 ? bit_of(row, q.w) : 0u);
-        } else {
+        k0 = i0 >= sj && i0 < ej;
+        k1 = i0 + 1 >= sj && i0 + 1 < ej;
+        k2 = i0 + 2 >= sj && i0 + 2 < ej;
+        k3 = i0 + 3 >= sj && i0 + 3 < ej;
+      }
+      // hub leaves: transposed bitmap probes (the row of id L + 32t is its loader lane's: (L >> 2) + 8t)
+      const bool hub = idx < tot && hidj >= 0;
+      if (!TDFS_TRANSPOSE && hub) {
+        const uint32_t* row = P.hub_bits + (long long)hidj * P.hub_words;
+        cnt += (k0 ? bit_of(row, q.x) : 0u) + (k1 ? bit_of(row, q.y) : 0u) + (k2 ? bit_of(row, q.z) : 0u) +
+               (k3 ? bit_of(row, q.w) : 0u);
+      } else if (TDFS_TRANSPOSE && __any_sync(FULL, hub)) {
+        reinterpret_cast<int4*>(tb)[lane] =
+            make_int4(hub && k0 ? q.x : -1, hub && k1 ? q.y : -1, hub && k2 ? q.z : -1, hub && k3 ? q.w : -1);
+        __syncwarp();
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+          const int w = tb[lane + 32 * t];
+          const int row = __shfl_sync(FULL, hidj, (lane >> 2) + 8 * t);
+          if (w >= 0) cnt += bit_of(P.hub_bits + (long long)row * P.hub_words, w);
+        }
+        __syncwarp();
+      }
+      if (idx < tot && hidj < 0) {
+        {
           // this lane's ids of one leaf increase group by group: search N(x_j) from the last hit;
           // ids outside the leaf's window search as +inf (they sit past every valid id)
           const int v0 = k0 ? q.x : INT_MAX, v1 = k1 ? q.y : INT_MAX, v2 = k2 ? q.z : INT_MAX, v3 = k3 ? q.w : INT_MAX;
@@ -644,6 +697,8 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     long long g0 = 0, sj = 0, ej = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
+      int4 q = make_int4(-1, -1, -1, -1);
+      bool k0 = false, k1 = false, k2 = false, k3 = false;
       if (idx < tot) {
         if (idx >= jn) {
           do { ++j; jn = pre[j + 1]; } while (jn <= idx);
@@ -657,16 +712,27 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
           fmaxj = F[hij - 1];
         }
         const long long g = g0 + idx - pj;
-        const int4 q = __ldg(adj4 + g);
+        q = __ldg(adj4 + g);
         const long long i0 = g << 2;
-        const bool k0 = i0 >= sj && i0 < ej && q.x >= fminj && q.x <= fmaxj;
-        const bool k1 = i0 + 1 >= sj && i0 + 1 < ej && q.y >= fminj && q.y <= fmaxj;
-        const bool k2 = i0 + 2 >= sj && i0 + 2 < ej && q.z >= fminj && q.z <= fmaxj;
-        const bool k3 = i0 + 3 >= sj && i0 + 3 < ej && q.w >= fminj && q.w <= fmaxj;
-        if (frow) {
-          cnt += (k0 ? bit_of(frow, q.x) : 0u) + (k1 ? bit_of(frow, q.y) : 0u) + (k2 ? bit_of(frow, q.z) : 0u) +
-                 (k3 ? bit_of(frow, q.w) : 0u);
-        } else {
+        k0 = i0 >= sj && i0 < ej && q.x >= fminj && q.x <= fmaxj;
+        k1 = i0 + 1 >= sj && i0 + 1 < ej && q.y >= fminj && q.y <= fmaxj;
+        k2 = i0 + 2 >= sj && i0 + 2 < ej && q.z >= fminj && q.z <= fmaxj;
+        k3 = i0 + 3 >= sj && i0 + 3 < ej && q.w >= fminj && q.w <= fmaxj;
+      }
+      if (!TDFS_TRANSPOSE && frow) {
+        cnt += (k0 ? bit_of(frow, q.x) : 0u) + (k1 ? bit_of(frow, q.y) : 0u) + (k2 ? bit_of(frow, q.z) : 0u) +
+               (k3 ? bit_of(frow, q.w) : 0u);
+      } else if (frow) {  // warp-uniform: transposed probes of y's bitmap
+        reinterpret_cast<int4*>(tb)[lane] = make_int4(k0 ? q.x : -1, k1 ? q.y : -1, k2 ? q.z : -1, k3 ? q.w : -1);
+        __syncwarp();
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+          const int w = tb[lane + 32 * t];
+          if (w >= 0) cnt += bit_of(frow, w);
+        }
+        __syncwarp();
+      } else if (idx < tot) {
+        {
           // F in shared memory: four lockstep searches; a kept id is <= F_max so its index is < hi
           int r0, r1, r2, r3;
           lower_bound4(F, loj, hij - loj, q.x, q.y, q.z, q.w, r0, r1, r2, r3);
@@ -681,7 +747,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
 // Stage F for the level-(k-2) list just built (see FRef).  Returns |F|, or -2 when F
 // would have to be materialised and exceeds the shared-memory stage (generic per leaf).
 template <bool STATS>
-__device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& fr) {
+__device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, FRef& fr) {
   const DevPlan& pl = P.plan;
   const int lane = c.lane;
   fr.F = c.sF;
@@ -711,21 +777,25 @@ __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, bool own2, FRef& 
       return (int)(b - a);
     }
   }
-  return (int)extend<3, STATS>(P, c, kVF, own2);
+  return (int)extend<3, STATS>(P, c, kVF);
 }
 
-// Push <S0, S1, L[2][i]> for i in [from, size) -- timeout split of level 2
-// (PAPER.md:268).  Returns the first index NOT pushed (size on success).
+// Push <S0, S1, L[2][i]> for i in [from, size) -- timeout split of level 2, one 3-prefix task
+// per remaining sibling.  Returns the first index NOT pushed (size on success).
 template <bool STATS>
 __device__ long long split_level2(const KParams& P, Ctx<STATS>& c, const Queue& q, long long from, long long size) {
   const uint32_t* table = c.tables;  // level index 0 = position 2
-  const int s0 = getS(c.sreg, 0), s1 = getS(c.sreg, 1);
+  Task k;
+  k.hdr = TASK_PREFIX;
+  k.v[0] = getS(c.sreg, 0);
+  k.v[1] = getS(c.sreg, 1);
+  k.v[3] = k.v[4] = k.v[5] = -1;
   for (long long base = from; base < size; base += 32) {
     const long long i = base + c.lane;
-    int v = 0;
-    if (i < size) v = paged_read(P, table, i);
+    k.v[2] = 0;
+    if (i < size) k.v[2] = paged_read(P, table, i);
     const unsigned mask = __ballot_sync(FULL, i < size);
-    if (!q_push_warp(P, q, mask, s0, s1, v, c.lane)) {
+    if (!q_push_warp(P, q, mask, k, c.lane)) {
       if (STATS && c.lane == 0) c.qfull++;
       return base;
     }
@@ -734,26 +804,32 @@ __device__ long long split_level2(const KParams& P, Ctx<STATS>& c, const Queue& 
   return size;
 }
 
-// Timeout split of level 2 when its children are leaves (k = 4): instead of one task per
-// remaining sibling (each a single Eq. (1) intersection), push at most 32 range tasks
-// <S0, S1, lo, hi>, each covering >= 32 consecutive siblings C[i .. i+g) by id range
-// [C[i], C[i+g]) (the last one up to this list's own bound w2hi).  A receiver rebuilds
-// its slice of level 2 with that extra window, stages the leaf set once and processes
-// the leaves in flat batches.  Returns false if the queue is full.
+// Timeout split of level d (2 <= d <= kMaxRangeLevel) into range tasks (R30/R33): instead
+// of one task per remaining sibling, push at most 32 tasks <S0 .. S_{d-1}, lo, hi>, each covering
+// >= 32 consecutive siblings C[i .. i+g) by id range [C[i], C[i+g]) (the last one up to this list's
+// own bound).  A receiver rebuilds that slice of level d (one more window bound), or the whole list
+// when a later position reuses it, and continues the DFS below it; it can time out and split its
+// slice again.  Returns false if the queue is full.
 template <bool STATS>
-__device__ bool split_level2_ranges(const KParams& P, Ctx<STATS>& c, const Queue& q, int from, int size) {
+__device__ bool split_ranges(const KParams& P, Ctx<STATS>& c, const Queue& q, int d, int from, int size) {
   const int lane = c.lane;
-  const uint32_t* table = c.tables;  // level index 0 = position 2
+  const uint32_t* table = c.tables + (size_t)(d - 2) * P.E;
   const int rem = size - from;
   const int g = max(kRangeMin, (rem + kRangeMaxT - 1) / kRangeMaxT);
   const int ntask = (rem + g - 1) / g;
   const int i0 = from + lane * g, i1 = i0 + g;
-  int lo = 0, hi = c.w2hi;
+  Task k;
+  k.hdr = TASK_RANGE | (d << 4);
+#pragma unroll
+  for (int i = 0; i < 6; i++) k.v[i] = getS(c.sreg, i);  // lanes >= d overwritten / unused
+  int lo = 0, hi = (c.wlev == d) ? c.whi : INT_MAX;
   if (lane < ntask) lo = paged_read(P, table, i0);
   if (lane < ntask && i1 < size) hi = paged_read(P, table, i1);
+#pragma unroll
+  for (int i = 2; i <= kMaxRangeLevel; i++)
+    if (i == d) { k.v[i] = lo; k.v[i + 1] = hi; }
   const unsigned mask = ntask >= 32 ? FULL : ((1u << ntask) - 1u);
-  const int s0 = getS(c.sreg, 0), s1 = getS(c.sreg, 1);
-  if (!q_push_warp(P, q, mask, s0, s1, lo, lane, hi)) {
+  if (!q_push_warp(P, q, mask, k, lane)) {
     if (STATS && lane == 0) c.qfull++;
     return false;
   }
@@ -767,10 +843,8 @@ template <int MODE, bool STATS>
 __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) {
   const int k = P.plan.k;
   const int lane = c.lane;
-  // level 2 built whole by this warp (not a <v1,v2,v3> task, not a range task's slice): reusable
-  const bool own2 = (start == 2) && c.w2mode != 1;
   if (start == k - 1) {
-    long long n = (MODE == 1) ? extend<2, STATS>(P, c, start, own2) : extend<1, STATS>(P, c, start, own2);
+    long long n = (MODE == 1) ? extend<2, STATS>(P, c, start) : extend<1, STATS>(P, c, start);
     c.count += (unsigned long long)n;
     return true;
   }
@@ -779,43 +853,44 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
   int nF = -1;  // staged |F|, -1 = not staged (generic Eq. (1) per leaf)
   FRef fr;
   int d = start;
-  long long sz = extend<0, STATS>(P, c, d, own2);
+  long long sz = extend<0, STATS>(P, c, d);
   if (sz < 0) return false;
   if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
-  if (start == 2 && c.w2mode == 2) {  // range task over a whole level-2 list: iterate [w2lo, w2hi) only
-    const long long ib = warp_paged_lower_bound(P, c.tables, 0, sz, c.w2lo, lane);
-    const long long ie = c.w2hi < INT_MAX ? warp_paged_lower_bound(P, c.tables, ib, sz, c.w2hi, lane) : sz;
+  if (start == c.wlev && c.wmode == 2) {  // range task over a whole list: iterate [wlo, whi) only
+    const uint32_t* tb = c.tables + (size_t)(d - 2) * P.E;
+    const long long ib = warp_paged_lower_bound(P, tb, 0, sz, c.wlo, lane);
+    const long long ie = c.whi < INT_MAX ? warp_paged_lower_bound(P, tb, ib, sz, c.whi, lane) : sz;
     if (lane == d) c.liter = (int)ib;
-    c.end2 = (int)ie;
+    c.wend = (int)ie;
   }
   if (use_lf && d == k - 2) {
-    nF = sz >= 2 ? stage_leaf_set(P, c, own2, fr) : -1;
+    nF = sz >= 2 ? stage_leaf_set(P, c, fr) : -1;
     if (nF == 0 && lane == d) c.liter = (int)sz;  // F empty: no leaf below this list
   }
-  bool grace = false;  // after a full queue: descend once in place before re-checking (progress for tau = 0)
+  int glev = 0;  // after a full queue at level glev: descend once in place before re-checking (progress at tau = 0)
   for (;;) {
     const int it = __shfl_sync(FULL, c.liter, d);
-    const int size = d == 2 ? min(__shfl_sync(FULL, c.lsize, d), c.end2) : __shfl_sync(FULL, c.lsize, d);
+    const int size = d == c.wlev ? min(__shfl_sync(FULL, c.lsize, d), c.wend) : __shfl_sync(FULL, c.lsize, d);
     if (it < size) {
-      if (d == 2 && !grace && timed_out(P, c)) {
+      if (((P.split_mask >> d) & 1u) && d != glev && timed_out(P, c)) {
         // timeout: push the current and all remaining siblings, then backtrack
         if (STATS && lane == 0) c.touts++;
-        if (k == 4 && P.range_split && P.range_ok) {
-          // <= 32 remaining siblings finish in place (tasks strictly shrink: progress at tau = 0)
+        if ((P.range_mask >> d) & 1u) {
+          // <= kRangeMin remaining siblings finish in place (tasks strictly shrink: progress at tau = 0)
           if (size - it <= kRangeMin) {
             if (lane == 0) c.t0 = globaltimer();
-            grace = true;
+            glev = d;
             continue;
           }
-          if (split_level2_ranges(P, c, q, it, size)) {
+          if (split_ranges(P, c, q, d, it, size)) {
             if (lane == d) c.liter = size;
             continue;
           }
           if (lane == 0) c.t0 = globaltimer();  // queue full: continue in place
-          grace = true;
+          glev = d;
           continue;
         }
-        long long upto = split_level2(P, c, q, it, size);
+        long long upto = split_level2(P, c, q, it, size);  // d == 2: the paper's per-sibling tasks
         if (upto >= size) {
           if (lane == d) c.liter = size;
           continue;
@@ -823,10 +898,10 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
         // queue full: the pushed prefix is gone, continue in place with t0 reset
         if (lane == d) c.liter = (int)upto;
         if (lane == 0) c.t0 = globaltimer();
-        grace = true;
+        glev = d;
         continue;
       }
-      if (d == 2) grace = false;
+      if (glev == d) glev = 0;
       const uint32_t* table = c.tables + (size_t)(d - 2) * P.E;
       if (d + 1 == k - 1 && use_lf && nF >= 0) {
         // staged leaves in batches of 32: the ids and N(x) metadata of the batch are
@@ -842,15 +917,15 @@ __device__ bool dfs(const KParams& P, Ctx<STATS>& c, const Queue& q, int start) 
       const int v = paged_read(P, table, it);
       if (lane == d) { c.sreg = v; c.liter = it + 1; }
       if (d + 1 == k - 1) {
-        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1, own2) : extend<1, STATS>(P, c, d + 1, own2);
+        long long n = (MODE == 1) ? extend<2, STATS>(P, c, d + 1) : extend<1, STATS>(P, c, d + 1);
         c.count += (unsigned long long)n;
       } else {
         d++;
-        sz = extend<0, STATS>(P, c, d, own2);
+        sz = extend<0, STATS>(P, c, d);
         if (sz < 0) return false;
         if (lane == d) { c.lsize = (int)sz; c.liter = 0; }
         if (use_lf && d == k - 2) {
-          nF = sz >= 2 ? stage_leaf_set(P, c, own2, fr) : -1;
+          nF = sz >= 2 ? stage_leaf_set(P, c, fr) : -1;
           if (nF == 0 && lane == d) c.liter = (int)sz;
         }
       }
@@ -903,10 +978,10 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
         if (lane == 0) ob0 = atomicAdd(ctr(P, C_OUTCUR), (unsigned long long)cnt);
         ob0 = __shfl_sync(FULL, ob0, 0);
         const unsigned long long idx = ob0 + __popc(mask & lanemask_lt());
-        if (ok && idx < P.cap) {
-          P.out[idx * 2 + pl.order[0]] = v0;
-          P.out[idx * 2 + pl.order[1]] = v1;
-        }
+        int t[kMaxK];
+        t[0] = v0;
+        t[1] = v1;
+        if (ok) emit_tuple(P, idx, t, 2);
       }
       c.count += (unsigned long long)cnt;
       continue;
@@ -915,7 +990,13 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
       // timeout check before descending into the next edge (edge level is split-eligible)
       if (timed_out(P, c)) {
         if (STATS && lane == 0) c.touts++;
-        if (q_push_warp(P, q, mask, v0, v1, -2, lane)) {
+        Task et;
+        et.hdr = TASK_EDGE;
+        et.v[0] = v0;
+        et.v[1] = v1;
+        et.v[2] = -2;
+        et.v[3] = et.v[4] = et.v[5] = -1;
+        if (q_push_warp(P, q, mask, et, lane)) {
           if (STATS && lane == 0) c.enq += __popc(mask);
           mask = 0;
           break;
@@ -952,10 +1033,12 @@ __global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(co
   c.t0 = 0;
   c.lnodes = 0;
   c.wbytes = c.sbytes = c.enq = c.deq = c.touts = c.qfull = c.scanned = c.edges_in = c.chunks = 0;
-  c.w2lo = 0;
-  c.w2hi = INT_MAX;
-  c.w2mode = 0;
-  c.end2 = INT_MAX;
+  c.wlev = 0;
+  c.wlo = 0;
+  c.whi = INT_MAX;
+  c.wmode = 0;
+  c.wend = INT_MAX;
+  c.own = 2;
   c.tables = P.page_tables + (size_t)gwarp * (size_t)max(P.n_levels, 1) * (size_t)P.E;
   c.sF = tdfs_smem + (threadIdx.x >> 5) * P.fcap;
   const Queue q = make_queue(P);
@@ -963,6 +1046,9 @@ __global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(co
   unsigned long long* cursor = P.gcursor;
 
   if (lane == 0) atomicAdd(active, 1);
+  const unsigned long long t_start = STATS ? globaltimer() : 0ull;
+  unsigned long long t_idle = t_start;
+  if (STATS && P.stats && lane == 0) atomicMin(P.stats + S_T_START, t_start);
   bool busy = true;
   for (;;) {
     if (read_error(P)) break;
@@ -987,32 +1073,46 @@ __global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(co
       busy = true;
     }
     // 1. Q_task first
-    int got = 0, t1 = 0, t2 = 0, t3 = 0, t4 = -1;
+    int got = 0;
+    Task tk;
     if (lane == 0) {
-      got = q_pop(q, t1, t2, t3, t4);
+      got = q_pop(q, tk);
       if (got) c.t0 = globaltimer();
     }
     got = __shfl_sync(FULL, got, 0);
     if (got) {
-      t1 = __shfl_sync(FULL, t1, 0);
-      t2 = __shfl_sync(FULL, t2, 0);
-      t3 = __shfl_sync(FULL, t3, 0);
-      t4 = __shfl_sync(FULL, t4, 0);
-      if (STATS && lane == 0) c.deq++;
-      if (lane == 0) c.sreg = t1;
-      if (lane == 1) c.sreg = t2;
-      if (lane == 2) c.sreg = t3;
-      const bool range = t3 >= 0 && t4 >= 0;  // <v1, v2, lo, hi>: level-2 candidates in [lo, hi)
-      if (range) {
-        c.w2lo = t3;
-        c.w2hi = t4;
-        c.w2mode = P.reuse2_used ? 2 : 1;
+      const int hdr = __shfl_sync(FULL, tk.hdr, 0);
+      int mine = 0;
+#pragma unroll
+      for (int i = 0; i < 6; i++) {
+        const int x = __shfl_sync(FULL, tk.v[i], 0);
+        if (lane == i) mine = x;
       }
-      const bool ok = dfs<MODE, STATS>(P, c, q, (t3 == -2 || range) ? 2 : 3);
-      c.w2lo = 0;
-      c.w2hi = INT_MAX;
-      c.w2mode = 0;
-      c.end2 = INT_MAX;
+      if (STATS && lane == 0) c.deq++;
+      const int kind = hdr & 15, lev = hdr >> 4;
+      int start = 2;
+      if (kind == TASK_EDGE) {
+        if (lane < 2) c.sreg = mine;
+      } else if (kind == TASK_PREFIX) {
+        if (lane < 3) c.sreg = mine;
+        start = 3;
+        c.own = 3;
+      } else {  // TASK_RANGE at level lev: prefix S[0 .. lev-1], ids [lo, hi)
+        if (lane < lev) c.sreg = mine;
+        c.wlev = lev;
+        c.wlo = __shfl_sync(FULL, mine, lev);
+        c.whi = __shfl_sync(FULL, mine, lev + 1);
+        c.wmode = ((P.reused_mask >> lev) & 1u) ? 2 : 1;
+        c.own = c.wmode == 2 ? lev : lev + 1;
+        start = lev;
+      }
+      const bool ok = dfs<MODE, STATS>(P, c, q, start);
+      c.wlev = 0;
+      c.wlo = 0;
+      c.whi = INT_MAX;
+      c.wmode = 0;
+      c.wend = INT_MAX;
+      c.own = 2;
       if (!ok) {
         raise_error(P, ERR_STACK);
         break;
@@ -1046,6 +1146,7 @@ __global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(co
     if (lane == 0) {
       __threadfence();
       atomicSub(active, 1);
+      if (STATS) t_idle = globaltimer();  // the last of these is when this warp's work ended
     }
     busy = false;
   }
@@ -1064,6 +1165,11 @@ __global__ void __launch_bounds__(kBlockThreads, TDFS_MIN_BLOCKS) tdfs_kernel(co
       atomicAdd(P.stats + S_EDGES_SCANNED, c.scanned);
       atomicAdd(P.stats + S_EDGES_IN, c.edges_in);
       atomicAdd(P.stats + S_CHUNKS, c.chunks);
+      const unsigned long long te = t_idle;  // load balance: when this warp last ran out of work
+      atomicMin(P.stats + S_T_EXIT_MIN, te);
+      atomicMax(P.stats + S_T_EXIT_MAX, te);
+      atomicAdd(P.stats + S_T_EXIT_SUM, te - t_start);
+      atomicAdd(P.stats + S_WARPS, 1ull);
     }
   }
 }
@@ -1074,7 +1180,8 @@ __global__ void init_queue_kernel(QSlot* slots, unsigned long long cap, unsigned
        s += (unsigned long long)gridDim.x * blockDim.x) {
     unsigned long long first = base + ((s + cap - (base % cap)) % cap);  // first ticket >= base hitting slot s
     slots[s].seq = (unsigned)first;
-    slots[s].v1 = slots[s].v2 = slots[s].v3 = slots[s].v4 = -1;
+    slots[s].hdr = -1;
+    for (int i = 0; i < 6; i++) slots[s].v[i] = -1;
   }
 }
 
@@ -1194,6 +1301,8 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   off += align_up(sizeof(unsigned long long) * C_NUM * kCounterStride, 256);
   L->stats = off;
   off += align_up(sizeof(unsigned long long) * S_NUM, 256);
+  L->fill = off;
+  off += align_up(sizeof(unsigned long long) * kRingChunks, 256);
   L->slots = off;
   off += align_up(sizeof(QSlot) * L->qslots, 256);
   L->tables = off;
@@ -1206,7 +1315,7 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
 
 int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
                int mode, int32_t* d_out, uint64_t cap, uint64_t* d_count, bool sync, uint64_t* h_count,
-               tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap, int64_t* n_trace) {
+               tdfs_stats* stats, int32_t* h_trace, int64_t trace_cap, int64_t* n_trace, bool ring) {
   WsLayout L;
   int rc = resolve_layout(g, p, o, &L);
   if (rc) return rc;
@@ -1232,12 +1341,23 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   }
   if (o->flags & TDFS_RUN_NO_SHORTCUT)
     for (int i = 0; i < kMaxK; i++) P.plan.shortcut[i] = 0;
-  P.reuse2_used = 0;  // does any later position (or the leaf set) start from position 2's list?
+  // lists reused by a later position or the leaf set: a range task over them builds them whole
+  P.reused_mask = 0;
   for (int i = 3; i <= kVF; i++)
-    if ((i < P.plan.k || i == kVF) && P.plan.reuse[i] == 2) P.reuse2_used = 1;
-  // range tasks rebuild level 2 per task: worth it unless the leaves are intersections that
-  // start from the splitter's level-2 list (k4: per-sibling tasks measured 86 vs 100 ms)
-  P.range_ok = !(P.reuse2_used && P.plan.lf_var);
+    if ((i < P.plan.k || i == kVF) && P.plan.reuse[i] >= 2) P.reused_mask |= 1u << P.plan.reuse[i];
+  // timeout splits (R30/R33): range tasks at levels 2 .. min(kMaxRangeLevel, k-2); the paper's
+  // per-sibling 3-prefix tasks at level 2 only with TDFS_RUN_NO_RANGE_TASKS.  A leaf-level list
+  // whose leaves start from its own C(d) (k4: reuse + lf_var) keeps per-sibling tasks at level 2:
+  // rebuilding it per range task costs more (measured 86 vs 100 ms).
+  P.split_mask = 1u << 2;  // level 2 always (its per-sibling split is the paper's)
+  P.range_mask = 0;
+  if (!(o->flags & TDFS_RUN_NO_RANGE_TASKS)) {
+    for (int d = 2; d <= std::min(kMaxRangeLevel, P.plan.k - 2); d++) {
+      const bool leaf_level_reused = d == P.plan.k - 2 && ((P.reused_mask >> d) & 1u) && P.plan.lf_var;
+      if (!leaf_level_reused) P.range_mask |= 1u << d;
+    }
+    P.split_mask |= P.range_mask;  // deeper levels split only into range tasks
+  }
   P.shard_rank = o->shard_rank;
   P.shard_world = o->shard_world;
   P.n_tasks = g->nnz > o->shard_rank ? (g->nnz - o->shard_rank + o->shard_world - 1) / o->shard_world : 0;
@@ -1271,7 +1391,6 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   P.tau_ns = o->tau_ns;
   P.fcap = (o->flags & TDFS_RUN_NO_LEAF_STAGE) ? 0 : L.fcap;
   P.meta_off = (int)smem_meta_offset(L.wpb, L.fcap);
-  P.range_split = (o->flags & TDFS_RUN_NO_RANGE_TASKS) ? 0 : 1;
   if (g->d_hub_bits && !(o->flags & TDFS_RUN_NO_HUB_BITMAP)) {
     P.hub_id = g->d_hub_id;
     P.hub_bits = g->d_hub_bits;
@@ -1279,6 +1398,11 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   }
   P.out = d_out;
   P.cap = cap;
+  if (ring) {
+    P.ring_nchunks = kRingChunks;
+    P.ring_chunk = cap / kRingChunks;
+    P.ring_fill = (unsigned long long*)(base + L.fill);
+  }
   int32_t* d_trace = nullptr;
   if (h_trace && trace_cap > 0) {
     if ((e = cudaMalloc(&d_trace, sizeof(int32_t) * 3 * (size_t)trace_cap)) != cudaSuccess)
@@ -1289,7 +1413,12 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
 
   const unsigned long long ticket_base = 0;
   init_counters_kernel<<<1, C_NUM * kCounterStride, 0, st>>>(P.ctr, P.qcap, ticket_base);
-  if (want_stats) cudaMemsetAsync(P.stats, 0, sizeof(unsigned long long) * S_NUM, st);
+  if (want_stats) {
+    cudaMemsetAsync(P.stats, 0, sizeof(unsigned long long) * S_NUM, st);
+    cudaMemsetAsync(P.stats + S_T_START, 0xff, sizeof(unsigned long long), st);   // min accumulators
+    cudaMemsetAsync(P.stats + S_T_EXIT_MIN, 0xff, sizeof(unsigned long long), st);
+  }
+  if (ring) cudaMemsetAsync(P.ring_fill, 0, sizeof(unsigned long long) * kRingChunks, st);
   {
     int nb = (int)std::min<uint64_t>((L.qslots + 255) / 256, 4096);
     init_queue_kernel<<<std::max(nb, 1), 256, 0, st>>>(P.slots, P.qslots, ticket_base);
@@ -1351,6 +1480,12 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     stats->pages_used = std::min<unsigned long long>(hc[C_POOL * kCounterStride], L.n_pages);
     stats->pool_pages = L.n_pages;
     stats->stream_bytes = hs[S_STREAM];
+    if (hs[S_WARPS]) {
+      const unsigned long long t0 = hs[S_T_START];
+      stats->warp_exit_first_ns = hs[S_T_EXIT_MIN] - t0;
+      stats->warp_exit_last_ns = hs[S_T_EXIT_MAX] - t0;
+      stats->warp_exit_mean_ns = hs[S_T_EXIT_SUM] / hs[S_WARPS];  // each warp from its own start (~t0)
+    }
     stats->grid_blocks = L.blocks;
     stats->warps_per_block = L.wpb;
     stats->page_table_entries = L.E;
@@ -1364,6 +1499,106 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
                                                 "(raise pool_bytes / page_table_entries); no count produced");
   if (h_count) *h_count = hc[C_COUNT * kCounterStride];
   if (mode == 1 && cap < hc[C_COUNT * kCounterStride]) return TDFS_E_OUTPUT_OVERFLOW;
+  return TDFS_OK;
+}
+
+
+// Streaming enumerate ("output S"): the kernel writes
+// tuples into a device ring of ring_cap tuples (kRingChunks chunks) and waits for free space;
+// this host loop copies every full chunk out on a side stream (the DMA engine, concurrent with
+// the persistent kernel), hands it to `sink`, zeroes the chunk's fill word and advances the
+// consumed counter the kernel waits on; after the kernel ends it drains the last partial chunks.
+int stream_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, size_t ws_bytes, void* stream,
+               int32_t* d_ring, uint64_t ring_cap, SinkFn sink, void* user, uint64_t* n_total) {
+  if (!sink || !d_ring || !n_total) return fail(TDFS_E_INVALID_ARG, "enumerate_stream: NULL ring, sink or n_total");
+  if (ring_cap < (uint64_t)kRingChunks || ring_cap % kRingChunks)
+    return fail(TDFS_E_INVALID_ARG, "enumerate_stream: ring_cap must be a positive multiple of 8");
+  const int k = p->k;
+  const uint64_t chunk = ring_cap / kRingChunks;
+  WsLayout L;
+  int rc = resolve_layout(g, p, o, &L);
+  if (rc) return rc;
+  cudaStream_t st = (cudaStream_t)stream, side = nullptr;
+  cudaEvent_t done = nullptr;
+  int32_t* host = nullptr;
+  unsigned long long* words = nullptr;  // pinned: [0] fill probe, [1] zero, [2] consumed
+  cudaError_t e = cudaSetDevice(g->device);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaHostAlloc(&host, sizeof(int32_t) * (size_t)(chunk * k), cudaHostAllocDefault);
+  if (e == cudaSuccess) e = cudaHostAlloc(&words, 4 * sizeof(unsigned long long), cudaHostAllocDefault);
+  auto cleanup = [&]() {
+    if (side) cudaStreamDestroy(side);
+    if (done) cudaEventDestroy(done);
+    if (host) cudaFreeHost(host);
+    if (words) cudaFreeHost(words);
+  };
+  if (e != cudaSuccess) {
+    cleanup();
+    return cuda_fail(e, "enumerate_stream: setup");
+  }
+  rc = launch_job(g, p, o, ws, ws_bytes, stream, 1, d_ring, ring_cap, nullptr, false, nullptr, nullptr, nullptr, 0,
+                  nullptr, true);
+  if (rc) {
+    cleanup();
+    return rc;
+  }
+  cudaEventRecord(done, st);
+  char* base = (char*)ws;
+  unsigned long long* d_fill = (unsigned long long*)(base + L.fill);
+  unsigned long long* d_ctr = (unsigned long long*)(base + L.ctr);
+  unsigned long long* d_consumed = d_ctr + C_CONSUMED * kCounterStride;
+  uint64_t consumed = 0;
+  bool aborted = false;
+  words[1] = 0;
+  auto deliver = [&](uint64_t n) -> cudaError_t {  // copy n tuples at `consumed` out, hand them to sink
+    const uint64_t slot = consumed % ring_cap;
+    cudaError_t x = cudaMemcpyAsync(host, d_ring + slot * k, sizeof(int32_t) * (size_t)(n * k), cudaMemcpyDeviceToHost, side);
+    if (x == cudaSuccess) x = cudaStreamSynchronize(side);
+    if (x == cudaSuccess && !aborted && sink(host, n, k, user) != 0) aborted = true;
+    return x;
+  };
+  for (;;) {
+    const int c = (int)((consumed / chunk) % kRingChunks);
+    e = cudaMemcpyAsync(words, d_fill + c, sizeof(unsigned long long), cudaMemcpyDeviceToHost, side);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(side);
+    if (e != cudaSuccess) break;
+    if (words[0] >= chunk) {  // chunk full: out, then free it for the kernel
+      if ((e = deliver(chunk)) != cudaSuccess) break;
+      consumed += chunk;
+      words[2] = aborted ? (1ull << 62) : consumed;  // abort: nobody waits any more (tuples dropped)
+      e = cudaMemcpyAsync(d_fill + c, words + 1, sizeof(unsigned long long), cudaMemcpyHostToDevice, side);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(d_consumed, words + 2, sizeof(unsigned long long), cudaMemcpyHostToDevice, side);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(side);
+      if (e != cudaSuccess) break;
+      continue;
+    }
+    const cudaError_t q = cudaEventQuery(done);
+    if (q == cudaSuccess) break;
+    if (q != cudaErrorNotReady) { e = q; break; }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+  if (e == cudaSuccess) e = cudaEventSynchronize(done);
+  unsigned long long hc[C_NUM * kCounterStride];
+  if (e == cudaSuccess) e = cudaMemcpy(hc, d_ctr, sizeof(hc), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) {
+    cleanup();
+    return cuda_fail(e, "enumerate_stream: kernel execution");
+  }
+  if (hc[C_ERROR * kCounterStride]) {
+    cleanup();
+    return fail(TDFS_E_STACK_EXHAUSTED, "stack page pool or page table exhausted; no output");
+  }
+  const uint64_t total = hc[C_OUTCUR * kCounterStride];
+  while (!aborted && consumed < total) {  // the job is over: every reserved slot is written
+    const uint64_t n = std::min<uint64_t>(chunk - consumed % chunk, total - consumed);
+    if ((e = deliver(n)) != cudaSuccess) break;
+    consumed += n;
+  }
+  cleanup();
+  if (e != cudaSuccess) return cuda_fail(e, "enumerate_stream: drain");
+  *n_total = total;
+  if (aborted) return fail(TDFS_E_INVALID_ARG, "enumerate_stream: the sink aborted (total still exact)");
   return TDFS_OK;
 }
 

@@ -96,21 +96,26 @@ __device__ __forceinline__ unsigned long long q_reserve(const Queue& q, int r) {
   return atomicAdd(q.tail, (unsigned long long)r);
 }
 
+// A task in registers (see QSlot).
+struct Task {
+  int hdr;
+  int v[6];
+};
+
 // one lane: write task into the slot of ticket t and publish it
-__device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, int v1, int v2, int v3, int v4) {
+__device__ __forceinline__ void q_publish(const Queue& q, unsigned long long t, const Task& k) {
   QSlot* s = q.slots + (t & (q.nslots - 1));
   unsigned want = (unsigned)t;
   while (ld_acquire_u32(&s->seq) != want) __nanosleep(32);
   volatile QSlot* vs = s;
-  vs->v1 = v1;
-  vs->v2 = v2;
-  vs->v3 = v3;
-  vs->v4 = v4;
+  vs->hdr = k.hdr;
+#pragma unroll
+  for (int i = 0; i < 6; i++) vs->v[i] = k.v[i];
   st_release_u32(&s->seq, (unsigned)(t + 1));
 }
 
 // lane 0: Alg. 3 dequeue.  Returns false when empty.
-__device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3, int& v4) {
+__device__ __forceinline__ bool q_pop(const Queue& q, Task& k) {
   if (ld_relaxed_s64(q.avail) <= 0) return false;
   long long old = (long long)atomicAdd(q.avail, (unsigned long long)(-1ll));
   if (old <= 0) {
@@ -122,19 +127,18 @@ __device__ __forceinline__ bool q_pop(const Queue& q, int& v1, int& v2, int& v3,
   unsigned want = (unsigned)(h + 1);
   while (ld_acquire_u32(&s->seq) != want) __nanosleep(32);
   volatile QSlot* vs = s;
-  v1 = vs->v1;
-  v2 = vs->v2;
-  v3 = vs->v3;
-  v4 = vs->v4;
+  k.hdr = vs->hdr;
+#pragma unroll
+  for (int i = 0; i < 6; i++) k.v[i] = vs->v[i];
   st_release_u32(&s->seq, (unsigned)(h + q.nslots));
   atomicAdd(q.free_, 1ull);
   return true;
 }
 
-// Warp-cooperative push of the tasks held by the lanes in `mask` (lane i pushes
-// <a_i, b_i, c_i, d_i>).  Returns false if the queue is full (nothing pushed).
-__device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, unsigned mask, int a, int b, int c,
-                                           int lane, int d = -1) {
+// Warp-cooperative push of the tasks held by the lanes in `mask` (lane i pushes its own task).
+// Returns false if the queue is full (nothing pushed).  The test trace records (v1, v2, v3) of
+// edge tasks as <v1, v2, -2> and of 3-prefix tasks as <v1, v2, v3>; range tasks as <v1, v2, -3 - d>.
+__device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, unsigned mask, const Task& k, int lane) {
   int r = __popc(mask);
   if (r == 0) return true;
   unsigned long long t = 0;
@@ -143,7 +147,7 @@ __device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, un
   if (t == ~0ull) return false;
   if (mask >> lane & 1u) {
     unsigned long long my = t + __popc(mask & lanemask_lt());
-    q_publish(q, my, a, b, c, d);
+    q_publish(q, my, k);
   }
   __syncwarp();
   if (P.trace) {
@@ -153,9 +157,10 @@ __device__ __forceinline__ bool q_push_warp(const KParams& P, const Queue& q, un
     if (mask >> lane & 1u) {
       unsigned long long i = base + __popc(mask & lanemask_lt());
       if ((long long)i < P.trace_cap) {
-        P.trace[3 * i] = a;
-        P.trace[3 * i + 1] = b;
-        P.trace[3 * i + 2] = c;
+        const int kind = k.hdr & 15;
+        P.trace[3 * i] = k.v[0];
+        P.trace[3 * i + 1] = k.v[1];
+        P.trace[3 * i + 2] = kind == TASK_EDGE ? -2 : kind == TASK_PREFIX ? k.v[2] : -3 - (k.hdr >> 4);
       }
     }
   }

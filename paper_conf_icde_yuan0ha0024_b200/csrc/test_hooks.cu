@@ -15,6 +15,16 @@ namespace {
 
 #include "prims.cuh"
 
+__device__ __forceinline__ Task mk_task(const int32_t* t3) {
+  Task k;
+  k.hdr = TASK_PREFIX;
+  k.v[0] = t3[0];
+  k.v[1] = t3[1];
+  k.v[2] = t3[2];
+  k.v[3] = k.v[4] = k.v[5] = -1;
+  return k;
+}
+
 // mode 0: one warp fills then drains; mode 1: n warps interleave push/pop then drain.
 __global__ void queue_test_kernel(KParams P, int mode, const int32_t* in, long long n_in, int32_t* out,
                                   unsigned long long* n_out, unsigned long long* n_enq) {
@@ -23,14 +33,15 @@ __global__ void queue_test_kernel(KParams P, int mode, const int32_t* in, long l
   const int nw = (gridDim.x * blockDim.x) >> 5;
   const Queue q = make_queue(P);
   auto pop_one = [&]() -> bool {
-    int got = 0, a = 0, b = 0, c = 0, d = 0;
-    if (lane == 0) got = q_pop(q, a, b, c, d);
+    int got = 0;
+    Task k;
+    if (lane == 0) got = q_pop(q, k);
     got = __shfl_sync(FULL, got, 0);
     if (got && lane == 0) {
       unsigned long long i = atomicAdd(n_out, 1ull);
-      out[3 * i] = a;
-      out[3 * i + 1] = b;
-      out[3 * i + 2] = c;
+      out[3 * i] = k.v[0];
+      out[3 * i + 1] = k.v[1];
+      out[3 * i + 2] = k.v[2];
     }
     return got != 0;
   };
@@ -38,7 +49,7 @@ __global__ void queue_test_kernel(KParams P, int mode, const int32_t* in, long l
     if (warp != 0) return;
     long long pushed = 0;
     for (long long i = 0; i < n_in; i++) {
-      bool ok = q_push_warp(P, q, 1u, in[3 * i], in[3 * i + 1], in[3 * i + 2], lane);
+      bool ok = q_push_warp(P, q, 1u, mk_task(in + 3 * i), lane);
       if (!ok) break;
       pushed++;
     }
@@ -53,7 +64,7 @@ __global__ void queue_test_kernel(KParams P, int mode, const int32_t* in, long l
     // push a batch of up to 32 consecutive tasks of this warp's stride when possible
     bool ok = false;
     while (!ok) {
-      ok = q_push_warp(P, q, 1u, in[3 * i], in[3 * i + 1], in[3 * i + 2], lane);
+      ok = q_push_warp(P, q, 1u, mk_task(in + 3 * i), lane);
       if (!ok) pop_one();
     }
     pushed++;
@@ -133,7 +144,8 @@ __global__ void init_q(QSlot* slots, unsigned long long cap, unsigned long long 
   for (unsigned long long s = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; s < nslots;
        s += (unsigned long long)gridDim.x * blockDim.x) {
     slots[s].seq = (unsigned)(base + ((s + nslots - (base % nslots)) % nslots));
-    slots[s].v1 = slots[s].v2 = slots[s].v3 = slots[s].v4 = -1;
+    slots[s].hdr = -1;
+    for (int i = 0; i < 6; i++) slots[s].v[i] = -1;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     ctrs[C_QHEAD * kCounterStride] = base;

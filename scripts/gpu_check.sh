@@ -6,8 +6,8 @@ TAG=${1:-x}
 K=${2:-}
 mkdir -p gpurun_out
 timeout 1800 python -m pytest tests -m gpu -q ${K:+-k "$K"} --timeout 600 --timeout-method=thread -p no:cacheprovider 2>&1 \
-  | grep -v "^  File\|^    " | tail -40 > gpurun_out/gputests_${TAG}.log
-tail -40 gpurun_out/gputests_${TAG}.log
+  > gpurun_out/gputests_${TAG}.log
+grep -E "^(FAILED|ERROR)|passed|failed" gpurun_out/gputests_${TAG}.log | tail -40
 timeout 900 python bench.py --steps 3 --warmup 3 --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err
 tail -3 gpurun_out/bench_${TAG}.err
 python - <<PY

@@ -69,41 +69,101 @@ def test_paged_write_ballot_compaction_and_min_page():
 
 
 # ------------------------------------------------------------------ Fig. 5 / Alg. 4
+def _level2_candidates(g, q, order, cons, v1, v2):
+    """Admissible f(pi_2) after the prefix (v1, v2), from the definition (sorted): adjacent to
+    the matched backward neighbours, distinct, inside the constraint window, degree filter of
+    DESIGN.md R8 (deg_Q(pi_2) > |B(pi_2)|)."""
+    nb = [set() for _ in range(g.n)]
+    for a, b in g.edges.tolist():
+        nb[a].add(b)
+        nb[b].add(a)
+    qadj = {(a, b) for a, b in q.edges} | {(b, a) for a, b in q.edges}
+    u = order[2]
+    S = [v1, v2]
+    back = [j for j in range(2) if (order[j], u) in qadj]
+    cand = set(range(g.n))
+    for j in back:
+        cand &= nb[S[j]]
+    cand -= {v1, v2}
+    pos = {w: i for i, w in enumerate(order)}
+    for a, b in cons:  # f(a) < f(b)
+        if pos[b] == 2 and pos[a] < 2:
+            cand = {x for x in cand if x > S[pos[a]]}
+        if pos[a] == 2 and pos[b] < 2:
+            cand = {x for x in cand if x < S[pos[b]]}
+    dq = sum(1 for a, b in q.edges if u in (a, b))
+    if dq > len(back):
+        cand = {x for x in cand if len(nb[x]) >= dq}
+    return sorted(cand)
+
+
 def test_timeout_split_single_warp_trace():
-    """tau = 0, one warp: every split-eligible step times out.  The trace must show
-    (a) the first chunk's edges pushed as <v1, v2, -2> in chunk order, (b) tasks never
-    carry more than 3 matched vertices, (c) every <v1,v2,v3> task
-    is an admissible 3-prefix, and the count is unchanged."""
-    g = T.rmat(9, 8, 5)
+    """Fig. 5 / Alg. 4 exactly, tau = 0, one warp, the paper's split rule
+    (TDFS_RUN_NO_RANGE_TASKS): the warp takes a chunk of 8 directed edges and, timing out before
+    the first descent, pushes the chunk's filtered-in edges as <v1, v2, -2> in CSR order; it then
+    dequeues them in FIFO order and, timing out at level 2 of each, pushes the current candidate and
+    all its siblings <v1, v2, v3> in ascending order; 3-prefix tasks (<= 3 matched vertices) are
+    never split further; then the next chunk.  The whole trace is derived from the definition."""
+    g = T.rmat(8, 6, 5)
     q = T.query("house")
     order = O.oracle_order(q)
+    cons = O.automorphisms(q)[1]
     h = U.load(g)
     p = U.plan(q, order, "auto")
-    o = M.default_opts(tau_ms=0.0, blocks=1, warps_per_block=1, chunk=8)
+    o = M.default_opts(tau_ms=0.0, blocks=1, warps_per_block=1, chunk=8, flags=M.TDFS_RUN_NO_RANGE_TASKS)
     cnt, trace, nt = M.tdfs_test_count_trace(h, p, o)
     assert cnt == O.count(g, q, "auto", order=order)
-    assert nt == trace.shape[0] > 0
-    two = trace[trace[:, 2] == -2]
-    three = trace[trace[:, 2] != -2]
-    assert two.shape[0] > 0 and three.shape[0] > 0
-    # (a) the first pushes are the first chunk's edges, in directed-edge (CSR) order:
-    # the leading run of 2-vertex tasks is strictly increasing in (v1, v2)
-    assert trace[0, 2] == -2
-    run = int(np.argmax(trace[:, 2] != -2)) if (trace[:, 2] != -2).any() else trace.shape[0]
-    keys = trace[:run, 0].astype(np.int64) * g.n + trace[:run, 1]
-    assert run >= 1 and (np.diff(keys) > 0).all()
-    # (c) 3-prefixes admissible: compare with the oracle's level-2 prefixes
-    sub_edges = [(a, b) for a, b in q.edges if a in order[:3] and b in order[:3]]
-    E = set(map(tuple, g.edges.tolist())) | {(b, a) for a, b in g.edges.tolist()}
-    qpos = {u: i for i, u in enumerate(order)}
-    for v1, v2, v3 in three[:5000]:
-        S = [int(v1), int(v2), int(v3)]
-        assert len(set(S)) == 3
-        for a, b in sub_edges:
-            assert (S[qpos[a]], S[qpos[b]]) in E
+    # expected: edge filter of positions 0, 1 (degree >= deg_Q, the (u1, u2) constraint)
+    offs, adj = T.to_csr(g)
+    deg = np.diff(offs)
+    src = np.repeat(np.arange(g.n), deg)
+    dq = [sum(1 for a, b in q.edges if u in (a, b)) for u in range(q.k)]
+    c01 = [(a, b) for a, b in cons if {a, b} == {order[0], order[1]}]
+    want = []
+    for c0 in range(0, adj.shape[0], 8):
+        edges = []
+        for e in range(c0, min(c0 + 8, adj.shape[0])):
+            v1, v2 = int(src[e]), int(adj[e])
+            if deg[v1] < dq[order[0]] or deg[v2] < dq[order[1]]:
+                continue
+            if any((a == order[0] and not v1 < v2) or (a == order[1] and not v2 < v1) for a, b in c01):
+                continue
+            edges.append((v1, v2))
+        want += [(v1, v2, -2) for v1, v2 in edges]
+        for v1, v2 in edges:
+            want += [(v1, v2, x) for x in _level2_candidates(g, q, order, cons, v1, v2)]
+    got = [tuple(int(x) for x in r) for r in trace]
+    assert nt == len(want)
+    assert got == want
     # every pushed task is dequeued exactly once
-    _, st = U.count(g, q, "auto", order=order, stats=True, tau_ms=0.0, blocks=1, warps_per_block=1)
+    _, st = U.count(g, q, "auto", order=order, stats=True, tau_ms=0.0, blocks=1, warps_per_block=1,
+                    flags=M.TDFS_RUN_NO_RANGE_TASKS)
     assert st["tasks_enqueued"] == st["tasks_dequeued"] == nt
+
+
+def test_deep_range_tasks_tau_zero():
+    """R33: with range tasks on (default) a timed-out level d (2 <= d <= min(4, k-2)) is split into
+    <= 32 id-range tasks <S0..S_{d-1}, lo, hi>; tau = 0 splits at every eligible step.  Counts,
+    per-level node counts and roofline bytes (STATS) still equal the oracle's for k = 5..7, every
+    pushed task is dequeued exactly once, and the trace shows range tasks at levels 3 and 4."""
+    g = T.rmat(8, 6, 8)  # w6: 18.5 M matches, 7.3 M level-5 prefixes
+    for name in ("house", "c5", "k5", "prism", "w6"):
+        q = T.query(name)
+        order = O.oracle_order(q)
+        r = O.match(g, q, "auto", order=order, deg_filter=True, threads=8)
+        for kw in (dict(tau_ms=0.0), dict(tau_ms=0.0, blocks=2, warps_per_block=2), dict(tau_ms=0.002)):
+            cnt, st = U.count(g, q, "auto", order=order, stats=True, **kw)
+            assert cnt == r["count"], (name, kw)
+            assert st["nodes_per_level"][1:q.k] == r["nodes"][1:q.k], (name, kw)
+            assert st["stream_bytes"] == r["W_stream"], (name, kw)
+            assert st["tasks_enqueued"] == st["tasks_dequeued"], (name, kw)
+            assert U.count(g, q, "auto", order=order, **kw) == r["count"], (name, kw)
+    q = T.query("w6")
+    h = U.load(g)
+    cnt, trace, nt = M.tdfs_test_count_trace(h, U.plan(q, O.oracle_order(q), "auto"),
+                                             M.default_opts(tau_ms=0.0, blocks=2, warps_per_block=2))
+    kinds = set(int(x) for x in trace[:, 2] if x < -2)
+    assert {-5, -6} <= kinds, kinds  # range tasks at levels 2 (-5), 3 (-6) and 4 (-7)
 
 
 def test_split_counts_are_tau_invariant_on_skewed_graph():

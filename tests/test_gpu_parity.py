@@ -143,6 +143,56 @@ def test_enumerate_chunks_stream_every_match_once(name, chunk_cap):
     assert np.array_equal(srt(np.concatenate(parts)), ref)
 
 
+@pytest.mark.parametrize("name,ring_cap", [("house", 8), ("house", 4096), ("c4", 64), ("k5", 8), ("edge", 16)])
+def test_enumerate_stream_tiny_ring_exact_set(name, ring_cap):
+    """NEXT-2 streaming enumerate: a ring far smaller than the output (warps wait for the host to
+    drain chunks, many wraps) still delivers exactly the oracle's match set, each match once."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    q = T.query(name)
+    g = T.rmat(8, 5, 4)
+    h = U.load(g)
+    ref = O.enumerate_sorted(g, q, "auto")
+    assert ref.shape[0] > 4 * ring_cap
+    parts = []
+    total = M.tdfs_enumerate_stream(h, U.plan(q), lambda a: parts.append(a), ring_cap,
+                                    M.default_opts(tau_ms=0.05))
+    got = np.concatenate(parts)
+    assert total == ref.shape[0] == got.shape[0]
+    assert np.array_equal(got[np.lexsort(got.T[::-1])], ref)
+    # a sink that stops early: the call reports it, the job still finishes
+    with pytest.raises(M.TdfsError):
+        M.tdfs_enumerate_stream(h, U.plan(q), lambda a: True, ring_cap)
+
+
+def test_enumerate_to_rank_local_files_config2_triangle(c2, tmp_path):
+    """NEXT-2 at scale: all 82.7 M triangles of config 2 streamed through a 2^20-tuple ring into two
+    rank-local files (shards 0 and 1 of 2); the union has the oracle golden's size, every row is a
+    triangle with f(u0) < f(u1) < f(u2) (C_auto) and no row repeats."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    gold = int(G.read("c2_counts.txt")["triangle"].split()[0])
+    h = U.load(c2)
+    p = M.plan_from_query(T.query("triangle"))
+    rows = []
+    for r in range(2):
+        path = str(tmp_path / f"tri_rank{r}.bin")
+        n = M.tdfs_enumerate_to_file(h, p, path, 1 << 20, M.default_opts(shard_rank=r, shard_world=2))
+        t = np.fromfile(path, dtype=np.int32).reshape(-1, 3)
+        assert t.shape[0] == n
+        rows.append(t)
+    t = np.concatenate(rows)
+    assert t.shape[0] == gold
+    assert (t[:, 0] < t[:, 1]).all() and (t[:, 1] < t[:, 2]).all()
+    offs, adj = T.to_csr(c2)
+    src = np.arange(c2.n, dtype=np.int64).repeat(np.diff(offs))
+    key = (src << 32) | adj.astype(np.int64)  # directed edge keys, sorted (CSR order)
+    for a, b in ((0, 1), (0, 2), (1, 2)):
+        kk = t[:, a].astype(np.int64) << 32 | t[:, b]
+        pos = np.searchsorted(key, kk)
+        assert (key[np.minimum(pos, key.shape[0] - 1)] == kk).all()
+    packed = (t[:, 0].astype(np.int64) << 36) | (t[:, 1].astype(np.int64) << 18) | t[:, 2]
+    assert np.unique(packed).shape[0] == gold
+
+
 def test_enumerate_overflow_keeps_exact_total():
     g = T.rmat(10, 8, 7)
     q = T.query("triangle")
