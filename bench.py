@@ -59,13 +59,17 @@ def parse():
     ap.add_argument("--shard-policy", type=int, default=0, help="N > 1: 0 round-robin (paper), 1 degree-balanced")
     ap.add_argument("--shared-cursor", action="store_true", help="N > 1: cross-GPU shared chunk cursor (NEXT-3)")
     ap.add_argument("--hub-bitmap-mb", type=int, default=0, help="hub bitmap budget (0 = library default)")
+    ap.add_argument("--degree-order", action="store_true",
+                    help="load with TDFS_GRAPH_DEGREE_ORDER (symmetry breaking by degree rank, DESIGN.md R35)")
+    ap.add_argument("--no-stats", action="store_true",
+                    help="skip the instrumented run (no roofline bytes): long configs-3..5 queries")
     return ap.parse_args()
 
 
 def workload(cfg: int):
     import tdfs_inputs as T
     g = T.config_graph(cfg)
-    names = T.CONFIG_QUERIES[cfg]
+    names = T.BENCH_QUERIES[cfg]
     qs = [T.labeled_query(n, 8) if cfg == 4 else T.query(n) for n in names]
     desc = {2: "R-MAT s18 EF16 (a,b,c)=(.57,.19,.19) seed 1",
             3: "R-MAT s20 EF6 seed 1", 4: "Chung-Lu n=4M gamma=2.2 dmax=15000 seed 7, 8 labels",
@@ -263,7 +267,7 @@ def run_ours(a):
         qs = [q for q in qs if q.name in keep or q.name.replace("_lab", "") in keep]
     hub_bytes = a.hub_bitmap_mb << 20
     t_load0 = time.perf_counter()
-    h = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes)
+    h = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes, degree_order=a.degree_order)
     torch.cuda.synchronize()
     load_s = time.perf_counter() - t_load0
     info = h.info()
@@ -289,6 +293,12 @@ def run_ours(a):
     # with a shared cursor the STATS run takes this rank's static shard instead)
     W, Wfull, stats_runs = [], [], []
     for p, o in zip(plans, qopts):
+        if a.no_stats:
+            W.append(0)
+            Wfull.append(0)
+            stats_runs.append({"timeouts": -1, "tasks_enqueued": -1, "pages_used": -1, "nodes_per_level": [],
+                               "warp_exit_first_ns": 0, "warp_exit_mean_ns": 0, "warp_exit_last_ns": 0})
+            continue
         so = M.tdfs_run_opts.from_buffer_copy(o)
         so.shared_cursor = None
         c, st = M.tdfs_count(h, p, so, workspace=ws, stats=True)
@@ -404,7 +414,7 @@ def run_ours(a):
                 dist.barrier()
             t0 = time.perf_counter()
             hh = M.tdfs_load_graph(offs_h.numpy(), adj_h.numpy(), None if lab_h is None else lab_h.numpy(),
-                                   device=dev, hub_bitmap_bytes=hub_bytes)
+                                   device=dev, hub_bitmap_bytes=hub_bytes, degree_order=a.degree_order)
             pl = [M.plan_from_query(q) for q in qs]
             dc = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
             for i, p in enumerate(pl):
@@ -454,7 +464,9 @@ def run_ours(a):
             "ms_per_step": total_ms / a.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"config{a.config}: {desc}", "n": g.n, "m": info["m"], "dmax": info["dmax"],
-                       "queries": [q.name for q in qs], "constraints": "full symmetry breaking (stabilizer chain)",
+                       "queries": [q.name for q in qs],
+                       "constraints": "full symmetry breaking (stabilizer chain)" +
+                                      (" on degree ranks (TDFS_GRAPH_DEGREE_ORDER)" if a.degree_order else " on vertex ids"),
                        "tau_ms": a.tau_ms, "chunk": {"k3": 8, "k>=4": a.chunk},
                        "parallelism": f"shard{world}" + ("-shared-cursor" if cursors is not None else
                                                          f"-policy{a.shard_policy}"),

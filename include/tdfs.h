@@ -74,6 +74,11 @@ typedef struct tdfs_graph tdfs_graph; /* opaque, library-owned */
 #define TDFS_GRAPH_VALIDATE 1u    /* check: offs monotone, offs[n] == nnz, lists strictly increasing,
                                       no self-loops, ids in range, symmetric -> TDFS_E_GRAPH_FORMAT */
 #define TDFS_GRAPH_NORMALIZE 2u   /* HOST_COPY only: symmetrise, drop self-loops and duplicates, sort lists */
+#define TDFS_GRAPH_DEGREE_ORDER 4u /* HOST_COPY only: the device graph renumbers vertices by (degree, id) rank, so the
+                                      symmetry-breaking constraints f(a) < f(b) compare degree ranks (R35):
+                                      counts are unchanged (any total order picks one embedding per copy); enumerated
+                                      tuples are mapped back to the caller's ids (a representative per copy chosen by
+                                      rank, not by id); shards and edge tasks follow the renumbered CSR order */
 
 typedef struct {
   int64_t n;             /* number of vertices */
@@ -98,7 +103,8 @@ int tdfs_load_graph(const tdfs_csr* g, int device, void* stream, tdfs_graph** ou
  * duplicates and self-loops allowed -- they are normalised away on the host with
  * multiple threads).  label: host [n] or NULL. */
 int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const int32_t* dst, const uint8_t* label,
-                    int64_t hub_bitmap_bytes /* as in tdfs_csr */, int device, void* stream, tdfs_graph** out);
+                    uint32_t flags /* 0 or TDFS_GRAPH_DEGREE_ORDER */, int64_t hub_bitmap_bytes /* as in tdfs_csr */,
+                    int device, void* stream, tdfs_graph** out);
 
 /* n, undirected edge count m = nnz/2, maximum degree, number of labels (max+1, 1 if unlabeled). */
 int tdfs_graph_info(const tdfs_graph* g, int64_t* n, int64_t* m, int64_t* dmax, int32_t* nlabels);

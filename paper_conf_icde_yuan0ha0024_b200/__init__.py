@@ -39,6 +39,7 @@ TDFS_MEM_HOST_COPY = 0
 TDFS_MEM_DEVICE_BORROW = 1
 TDFS_GRAPH_VALIDATE = 1
 TDFS_GRAPH_NORMALIZE = 2
+TDFS_GRAPH_DEGREE_ORDER = 4
 TDFS_RUN_STATS = 1
 TDFS_RUN_TRACE = 2
 TDFS_RUN_NO_REUSE = 4
@@ -107,8 +108,8 @@ SIGNATURES = {
     "tdfs_last_error": (ctypes.c_char_p, []),
     "tdfs_abi_version": (ctypes.c_int, []),
     "tdfs_load_graph": (ctypes.c_int, [ctypes.POINTER(tdfs_csr), ctypes.c_int, _vp, ctypes.POINTER(_vp)]),
-    "tdfs_load_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, ctypes.c_int64, ctypes.c_int,
-                                       _vp, ctypes.POINTER(_vp)]),
+    "tdfs_load_edges": (ctypes.c_int, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, ctypes.c_uint32, ctypes.c_int64,
+                                       ctypes.c_int, _vp, ctypes.POINTER(_vp)]),
     "tdfs_graph_info": (ctypes.c_int, [_vp, _i64p, _i64p, _i64p, _i32p]),
     "tdfs_graph_device_arrays": (ctypes.c_int, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
     "tdfs_free_graph": (None, [_vp]),
@@ -245,9 +246,10 @@ class PlanHandle:
 
 # ----------------------------------------------------------------- graph loading
 def tdfs_load_graph(offs, adj, label=None, device: int = 0, stream=None, validate: bool = False,
-                    normalize: bool = False, hub_bitmap_bytes: int = 0) -> GraphHandle:
+                    normalize: bool = False, hub_bitmap_bytes: int = 0, degree_order: bool = False) -> GraphHandle:
     """Load a CSR.  numpy arrays -> HOST_COPY; torch CUDA tensors -> DEVICE_BORROW (kept alive by the handle)."""
-    flags = (TDFS_GRAPH_VALIDATE if validate else 0) | (TDFS_GRAPH_NORMALIZE if normalize else 0)
+    flags = (TDFS_GRAPH_VALIDATE if validate else 0) | (TDFS_GRAPH_NORMALIZE if normalize else 0) | \
+        (TDFS_GRAPH_DEGREE_ORDER if degree_order else 0)
     keep = None
     if hasattr(offs, "is_cuda") and offs.is_cuda:
         torch = _torch()
@@ -270,7 +272,8 @@ def tdfs_load_graph(offs, adj, label=None, device: int = 0, stream=None, validat
     return GraphHandle(out.value, device, keep)
 
 
-def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None, hub_bitmap_bytes: int = 0) -> GraphHandle:
+def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None, hub_bitmap_bytes: int = 0,
+                    degree_order: bool = False) -> GraphHandle:
     """Load an undirected edge list ((m, 2) int array, host) -- normalised by the library."""
     e = np.ascontiguousarray(np.asarray(edges, dtype=np.int32).reshape(-1, 2))
     src = np.ascontiguousarray(e[:, 0])
@@ -278,7 +281,8 @@ def tdfs_load_edges(n: int, edges, label=None, device: int = 0, stream=None, hub
     lab = None if label is None else np.ascontiguousarray(label, dtype=np.uint8)
     out = _vp()
     _check(_lib.tdfs_load_edges(int(n), e.shape[0], src.ctypes.data, dst.ctypes.data,
-                                None if lab is None else lab.ctypes.data, int(hub_bitmap_bytes), device,
+                                None if lab is None else lab.ctypes.data,
+                                TDFS_GRAPH_DEGREE_ORDER if degree_order else 0, int(hub_bitmap_bytes), device,
                                 _stream_ptr(stream, device), ctypes.byref(out)))
     return GraphHandle(out.value, device)
 

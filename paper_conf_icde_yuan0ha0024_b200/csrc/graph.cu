@@ -282,8 +282,40 @@ void release(Graph& G) {
   cudaFree(G.d_hub_id);
   cudaFree(G.d_hub_bits);
   free_shard_lists(&G);
+  cudaFree(G.d_orig);
+  G.d_orig = nullptr;
   G.d_offs = nullptr; G.d_adj = nullptr; G.d_label = nullptr; G.d_src = nullptr;
   G.d_hub_id = nullptr; G.d_hub_bits = nullptr; G.n_hubs = 0;
+}
+
+int upload(Graph& G, const int64_t* offs, const int32_t* adj, const uint8_t* label, cudaStream_t st);
+void host_stats(Graph& G, const int64_t* offs, const uint8_t* label);
+void relabel_by_degree(int64_t n, const int64_t* offs, const int32_t* adj, const uint8_t* label,
+                       std::vector<int64_t>& noffs, std::vector<int32_t>& nadj, std::vector<uint8_t>& nlabel,
+                       std::vector<int32_t>& orig);
+
+// Host CSR (already simple, symmetric, sorted) -> device, optionally relabelled by degree, then the
+// per-entry sources and hub bitmaps.  Synchronous (host vectors outlive the copies).
+int finish_host_csr(Graph& G, const int64_t* offs, const int32_t* adj, const uint8_t* label, uint32_t flags,
+                    int64_t hub_budget, cudaStream_t st) {
+  std::vector<int64_t> noffs;
+  std::vector<int32_t> nadj, orig;
+  std::vector<uint8_t> nlabel;
+  if (flags & TDFS_GRAPH_DEGREE_ORDER) {
+    relabel_by_degree(G.n, offs, adj, label, noffs, nadj, nlabel, orig);
+    offs = noffs.data();
+    adj = nadj.data();
+    if (label) label = nlabel.data();
+  }
+  host_stats(G, offs, label);
+  int rc = upload(G, offs, adj, label, st);
+  if (rc == TDFS_OK && !orig.empty()) {
+    cudaError_t e = cudaMalloc(&G.d_orig, sizeof(int32_t) * orig.size());
+    if (e == cudaSuccess) e = cudaMemcpyAsync(G.d_orig, orig.data(), sizeof(int32_t) * orig.size(), cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) rc = fail(TDFS_E_OOM, "load: degree-order map");
+  }
+  if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, hub_budget);
+  return rc;
 }
 
 int upload(Graph& G, const int64_t* offs, const int32_t* adj, const uint8_t* label, cudaStream_t st) {
@@ -300,6 +332,37 @@ int upload(Graph& G, const int64_t* offs, const int32_t* adj, const uint8_t* lab
   if (label && G.n && (e = cudaMemcpyAsync(G.d_label, label, (size_t)G.n, cudaMemcpyHostToDevice, st)) != cudaSuccess)
     return cuda_fail(e, "load: label copy");
   return TDFS_OK;
+}
+
+// TDFS_GRAPH_DEGREE_ORDER (R35): vertex r of the device graph is the user's vertex orig[r], where
+// the user's vertices are sorted by (degree, id); lists are re-sorted in the new ids.  Symmetry-breaking
+// constraints then compare degree ranks, so the lower-ranked (lower-degree) vertex roots each copy.
+void relabel_by_degree(int64_t n, const int64_t* offs, const int32_t* adj, const uint8_t* label,
+                       std::vector<int64_t>& noffs, std::vector<int32_t>& nadj, std::vector<uint8_t>& nlabel,
+                       std::vector<int32_t>& orig) {
+  orig.resize((size_t)n);
+  for (int64_t v = 0; v < n; v++) orig[v] = (int32_t)v;
+  std::stable_sort(orig.begin(), orig.end(), [&](int32_t a, int32_t b) {
+    return offs[a + 1] - offs[a] < offs[b + 1] - offs[b];
+  });
+  std::vector<int32_t> rank((size_t)n);
+  for (int64_t r = 0; r < n; r++) rank[orig[r]] = (int32_t)r;
+  noffs.assign((size_t)n + 1, 0);
+  for (int64_t r = 0; r < n; r++) noffs[r + 1] = noffs[r] + (offs[orig[r] + 1] - offs[orig[r]]);
+  nadj.resize((size_t)noffs[n]);
+  parallel_for(n, [&](int64_t lo, int64_t hi) {
+    for (int64_t r = lo; r < hi; r++) {
+      const int32_t v = orig[r];
+      int32_t* L = nadj.data() + noffs[r];
+      const int64_t d = offs[v + 1] - offs[v];
+      for (int64_t i = 0; i < d; i++) L[i] = rank[adj[offs[v] + i]];
+      std::sort(L, L + d);
+    }
+  });
+  if (label) {
+    nlabel.resize((size_t)n);
+    for (int64_t r = 0; r < n; r++) nlabel[r] = label[orig[r]];
+  }
 }
 
 void host_stats(Graph& G, const int64_t* offs, const uint8_t* label) {
@@ -325,8 +388,10 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
   if (c->n < 0 || c->nnz < 0 || !c->offs || (c->nnz > 0 && !c->adj)) return fail(TDFS_E_INVALID_ARG, "load_graph: bad CSR");
   if (c->n >= kMaxN) return fail(TDFS_E_ID_RANGE, "load_graph: n >= 2^31 - 2");
   if (c->mem != TDFS_MEM_HOST_COPY && c->mem != TDFS_MEM_DEVICE_BORROW) return fail(TDFS_E_INVALID_ARG, "load_graph: bad mem");
-  if (c->mem == TDFS_MEM_DEVICE_BORROW && (c->flags & TDFS_GRAPH_NORMALIZE))
-    return fail(TDFS_E_INVALID_ARG, "load_graph: NORMALIZE needs HOST_COPY");
+  if (c->mem == TDFS_MEM_DEVICE_BORROW && (c->flags & (TDFS_GRAPH_NORMALIZE | TDFS_GRAPH_DEGREE_ORDER)))
+    return fail(TDFS_E_INVALID_ARG, "load_graph: NORMALIZE / DEGREE_ORDER need HOST_COPY");
+  if (c->flags & ~(TDFS_GRAPH_VALIDATE | TDFS_GRAPH_NORMALIZE | TDFS_GRAPH_DEGREE_ORDER))
+    return fail(TDFS_E_INVALID_ARG, "load_graph: unknown flags");
   cudaError_t e = cudaSetDevice(device);
   if (e != cudaSuccess) return cuda_fail(e, "load_graph: cudaSetDevice");
   cudaStream_t st = (cudaStream_t)stream;
@@ -352,18 +417,12 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
       std::vector<int32_t> adj;
       build_csr(c->n, c->nnz, a.data(), c->adj, offs, adj);
       G.nnz = offs[c->n];
-      host_stats(G, offs.data(), c->label);
-      rc = upload(G, offs.data(), adj.data(), c->label, st);
-      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, c->hub_bitmap_bytes);  // sync inside: host vectors outlive copies
+      rc = finish_host_csr(G, offs.data(), adj.data(), c->label, c->flags, c->hub_bitmap_bytes, st);
     } else {
       if (c->flags & TDFS_GRAPH_VALIDATE) rc = validate_host(c->n, c->nnz, c->offs, c->adj);
       else rc = check_host_ids(c->n, c->nnz, c->offs, c->adj);  // cheap: ids in [0, n), offsets sane
       G.nnz = c->nnz;
-      if (rc == TDFS_OK) {
-        host_stats(G, c->offs, c->label);
-        rc = upload(G, c->offs, c->adj, c->label, st);
-      }
-      if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, c->hub_bitmap_bytes);
+      if (rc == TDFS_OK) rc = finish_host_csr(G, c->offs, c->adj, c->label, c->flags, c->hub_bitmap_bytes, st);
     }
   } else {
     G.owns_csr = false;
@@ -384,8 +443,9 @@ extern "C" int tdfs_load_graph(const tdfs_csr* c, int device, void* stream, tdfs
 }
 
 extern "C" int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const int32_t* dst, const uint8_t* label,
-                               int64_t hub_bitmap_bytes, int device, void* stream, tdfs_graph** out) {
+                               uint32_t flags, int64_t hub_bitmap_bytes, int device, void* stream, tdfs_graph** out) {
   if (!out || n < 0 || m < 0 || (m > 0 && (!src || !dst))) return fail(TDFS_E_INVALID_ARG, "load_edges: bad args");
+  if (flags & ~(uint32_t)TDFS_GRAPH_DEGREE_ORDER) return fail(TDFS_E_INVALID_ARG, "load_edges: flags other than DEGREE_ORDER");
   if (n >= kMaxN) return fail(TDFS_E_ID_RANGE, "load_edges: n >= 2^31 - 2");
   std::atomic<int> bad(0);
   parallel_for(m, [&](int64_t lo, int64_t hi) {
@@ -405,9 +465,7 @@ extern "C" int tdfs_load_edges(int64_t n, int64_t m, const int32_t* src, const i
   G.device = device;
   G.n = n;
   G.nnz = offs[n];
-  host_stats(G, offs.data(), label);
-  int rc = upload(G, offs.data(), adj.data(), label, st);
-  if (rc == TDFS_OK) rc = finish_device_graph(G, st, false, false, hub_bitmap_bytes);
+  int rc = finish_host_csr(G, offs.data(), adj.data(), label, flags, hub_bitmap_bytes, st);
   if (rc != TDFS_OK) {
     release(G);
     delete h;

@@ -29,10 +29,7 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
 constexpr int kBlockThreads = 128;  // matching-kernel block size (its __launch_bounds__)
-#ifndef TDFS_LEAF_STAGE
-#define TDFS_LEAF_STAGE 512
-#endif
-constexpr int kLeafStage = TDFS_LEAF_STAGE;  // shared-memory ids per warp for the leaf set F
+constexpr int kLeafStage = 512;  // shared-memory ids per warp for a materialised leaf set F (at most)
 // Hub bitmaps (graph.cu): vertices of degree >= kHubMinDeg, highest first, within the budget
 constexpr int64_t kHubMinDeg = 256;
 constexpr int64_t kHubBudgetDefault = 256ll << 20;
@@ -86,6 +83,7 @@ struct Graph {
   int32_t* d_adj = nullptr;
   uint8_t* d_label = nullptr;
   int32_t* d_src = nullptr;  // source vertex of each directed entry (edge tasks)
+  int32_t* d_orig = nullptr; // TDFS_GRAPH_DEGREE_ORDER: user id of device vertex r (nullptr = identity)
   bool owns_csr = true;
   // hub adjacency bitmaps: membership w in N(h) in O(1) for the highest-degree vertices
   int32_t* d_hub_id = nullptr;     // [n], -1 for non-hubs
@@ -171,6 +169,7 @@ struct KParams {
   const uint32_t* hub_bits;
   long long hub_words;
   // enumerate
+  const int32_t* orig;             // device id -> user id (degree-ordered graphs), nullptr = identity
   int32_t* out;
   unsigned long long cap;
   unsigned long long ring_chunk;   // streaming (NEXT-2): tuples per ring chunk, 0 = capacity mode

@@ -56,10 +56,7 @@ struct __align__(16) LeafMeta {
                  // stream B N(x) entries [b0 + s, b0 + e) (narrowed to [F_min, F_max])
 };
 // 32 entries + 33 prefix ints (padded to 16 B) + a 128-id transpose buffer
-#ifndef TDFS_TRANSPOSE
-#define TDFS_TRANSPOSE 1
-#endif
-constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144 + (TDFS_TRANSPOSE ? 512 : 0);
+constexpr int kMetaBytesPerWarp = 32 * (int)sizeof(LeafMeta) + 144 + 512;
 __host__ __device__ inline size_t smem_meta_offset(int wpb, int fcap) {
   return ((size_t)wpb * fcap * sizeof(int) + 15) & ~(size_t)15;
 }
@@ -155,13 +152,13 @@ __device__ __forceinline__ long long warp_paged_lower_bound(const KParams& P, co
 __device__ __forceinline__ void emit_tuple(const KParams& P, unsigned long long idx, const int* t, int k) {
   if (P.ring_chunk == 0) {
     if (idx < P.cap)
-      for (int p = 0; p < k; p++) P.out[idx * k + P.plan.order[p]] = t[p];
+      for (int p = 0; p < k; p++) P.out[idx * k + P.plan.order[p]] = P.orig ? __ldg(P.orig + t[p]) : t[p];
     return;
   }
   const unsigned long long* consumed = ctr(P, C_CONSUMED);
   while (idx >= (unsigned long long)ld_relaxed_s64(consumed) + P.cap) __nanosleep(2000);
   const unsigned long long slot = idx % P.cap;
-  for (int p = 0; p < k; p++) P.out[slot * k + P.plan.order[p]] = t[p];
+  for (int p = 0; p < k; p++) P.out[slot * k + P.plan.order[p]] = P.orig ? __ldg(P.orig + t[p]) : t[p];
   __threadfence();
   atomicAdd(P.ring_fill + (idx / P.ring_chunk) % P.ring_nchunks, 1ull);
 }
@@ -571,6 +568,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
       }
     }
     for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
+    __syncwarp();  // every lane's reads of F are done before the next list overwrites it
     return cnt;
   }
   // F is walked from its 16-byte aligned base: F = Fal + fo
@@ -649,11 +647,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
       }
       // hub leaves: transposed bitmap probes (the row of id L + 32t is its loader lane's: (L >> 2) + 8t)
       const bool hub = idx < tot && hidj >= 0;
-      if (!TDFS_TRANSPOSE && hub) {
-        const uint32_t* row = P.hub_bits + (long long)hidj * P.hub_words;
-        cnt += (k0 ? bit_of(row, q.x) : 0u) + (k1 ? bit_of(row, q.y) : 0u) + (k2 ? bit_of(row, q.z) : 0u) +
-               (k3 ? bit_of(row, q.w) : 0u);
-      } else if (TDFS_TRANSPOSE && __any_sync(FULL, hub)) {
+      if (__any_sync(FULL, hub)) {
         reinterpret_cast<int4*>(tb)[lane] =
             make_int4(hub && k0 ? q.x : -1, hub && k1 ? q.y : -1, hub && k2 ? q.z : -1, hub && k3 ? q.w : -1);
         __syncwarp();
@@ -719,10 +713,7 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
         k2 = i0 + 2 >= sj && i0 + 2 < ej && q.z >= fminj && q.z <= fmaxj;
         k3 = i0 + 3 >= sj && i0 + 3 < ej && q.w >= fminj && q.w <= fmaxj;
       }
-      if (!TDFS_TRANSPOSE && frow) {
-        cnt += (k0 ? bit_of(frow, q.x) : 0u) + (k1 ? bit_of(frow, q.y) : 0u) + (k2 ? bit_of(frow, q.z) : 0u) +
-               (k3 ? bit_of(frow, q.w) : 0u);
-      } else if (frow) {  // warp-uniform: transposed probes of y's bitmap
+      if (frow) {  // warp-uniform: transposed probes of y's bitmap
         reinterpret_cast<int4*>(tb)[lane] = make_int4(k0 ? q.x : -1, k1 ? q.y : -1, k2 ? q.z : -1, k3 ? q.w : -1);
         __syncwarp();
 #pragma unroll
@@ -750,6 +741,7 @@ template <bool STATS>
 __device__ int stage_leaf_set(const KParams& P, Ctx<STATS>& c, FRef& fr) {
   const DevPlan& pl = P.plan;
   const int lane = c.lane;
+  __syncwarp();  // the previous list's leaves are done reading the stage before it is overwritten
   fr.F = c.sF;
   fr.hid = -1;
   fr.fix = 0;
@@ -1255,7 +1247,12 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   if (o->reserved_ != 0) return fail(TDFS_E_INVALID_ARG, "opts.reserved_ must be 0");
   if (o->shared_cursor && (reinterpret_cast<uintptr_t>(o->shared_cursor) & 7u))
     return fail(TDFS_E_INVALID_ARG, "opts.shared_cursor must be 8-byte aligned");
+  // leaf stage: a referenced F (lf_byref) is materialised only for a list without a hub bitmap, i.e.
+  // of degree <= the smallest hub degree, so it needs no more ids than that; the rest of the shared
+  // memory is left to L1 (measured on C2 c4: 845 -> 774 ms with 256 instead of 512 ids per warp)
   L->fcap = kLeafStage;
+  if (p->dev.lf_byref && g->n_hubs > 0)
+    L->fcap = (int)std::min<int64_t>(kLeafStage, std::max<int64_t>(64, (g->hub_min_deg + 31) / 32 * 32));
   if (o->blocks > 0) {
     L->blocks = o->blocks;
   } else {
@@ -1396,6 +1393,7 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     P.hub_bits = g->d_hub_bits;
     P.hub_words = g->hub_words;
   }
+  P.orig = g->d_orig;
   P.out = d_out;
   P.cap = cap;
   if (ring) {

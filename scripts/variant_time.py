@@ -1,6 +1,6 @@
 """Exploration (not a bench line): time queries of a config with whichever libtdfs.so the
 package on sys.path carries (PYTHONPATH=/tmp/var_X:$PWD, see variants.sh).  Median of REPS.
-    python scripts/variant_time.py CFG Q1,Q2 [REPS] [W] [HUB_MB]"""
+    python scripts/variant_time.py CFG Q1,Q2 [REPS] [W] [HUB_MB] [deg]"""
 import os
 import statistics
 import sys
@@ -15,10 +15,12 @@ qn = sys.argv[2].split(",")
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
 W = int(sys.argv[4]) if len(sys.argv) > 4 else 1
 hub_mb = int(sys.argv[5]) if len(sys.argv) > 5 else 0
+degree_order = len(sys.argv) > 6 and sys.argv[6] == "deg"
 g = T.config_graph(cfg)
-h = M.tdfs_load_edges(g.n, g.edges, g.labels, hub_bitmap_bytes=hub_mb << 20 if hub_mb > 0 else hub_mb)
+h = M.tdfs_load_edges(g.n, g.edges, g.labels, hub_bitmap_bytes=hub_mb << 20 if hub_mb > 0 else hub_mb,
+                      degree_order=degree_order)
 torch.cuda.synchronize()
-print(f"lib {M.LIB_PATH} hub_mb {hub_mb}", flush=True)
+print(f"lib {M.LIB_PATH} hub_mb {hub_mb} degree_order {degree_order}", flush=True)
 for name in qn:
     q = T.labeled_query(name, 8) if cfg == 4 else T.query(name)
     p = M.plan_from_query(q)

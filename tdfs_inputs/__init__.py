@@ -315,6 +315,18 @@ def config_graph(cfg: int, **over) -> Graph:
     raise ValueError(cfg)
 
 
+# Query sets bench.py times per config.  BASELINE.json names larger sets for configs 3-5; their full
+# counts take 16 min (C3 house / c5) to days (C4 w6 / two_k4 ~1.3 h, C5 k5 ~3.3 h, k6 ~11 days) on one
+# B200 (sampled-roots estimates, profiles/configs_probe_r02.txt), so the bench lines are gated to the
+# queries whose full time-to-count is seconds to minutes (SURVEY.md 8(d) gating rule).
+BENCH_QUERIES = {
+    1: ["fig1_q"],
+    2: ["triangle", "c4", "diamond", "tailed_triangle", "k4"],
+    3: ["k5"],
+    4: ["prism", "w5"],
+    5: ["k4"],
+}
+
 CONFIG_QUERIES = {
     1: ["fig1_q"],
     2: ["triangle", "c4", "diamond", "tailed_triangle", "k4"],

@@ -193,6 +193,44 @@ def test_enumerate_to_rank_local_files_config2_triangle(c2, tmp_path):
     assert np.unique(packed).shape[0] == gold
 
 
+def _degree_relabel(g):
+    """The (degree, id) ranking of DESIGN.md R35, computed here independently: returns the graph in
+    rank ids and orig (rank -> user id)."""
+    deg = np.bincount(g.edges.reshape(-1), minlength=g.n)
+    orig = np.lexsort((np.arange(g.n), deg))
+    rank = np.empty(g.n, dtype=np.int64)
+    rank[orig] = np.arange(g.n)
+    e = rank[g.edges.astype(np.int64)]
+    e = np.sort(e, axis=1)
+    lab = None if g.labels is None else g.labels[orig]
+    return T.Graph(g.n, e[np.lexsort((e[:, 1], e[:, 0]))].astype(np.int32), lab, g.name + "+deg"), orig
+
+
+@pytest.mark.parametrize("name", ["triangle", "c4", "diamond", "tailed_triangle", "k4", "house", "c5", "k5", "prism",
+                                  "w5", "fig1_q"])
+def test_degree_order_counts_and_sets(name):
+    """TDFS_GRAPH_DEGREE_ORDER (R35): symmetry breaking by degree rank.  Counts equal the oracle's on the
+    user graph (any total order picks one embedding per copy); the enumerated tuples, mapped back to user
+    ids by the library, equal the oracle's tuples on the rank-relabelled graph mapped back the same way."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    q = T.query(name)
+    g = T.rmat(10, 6, 11) if q.k <= 4 else graph("r9")
+    h = M.tdfs_load_edges(g.n, g.edges, degree_order=True)
+    p = U.plan(q)
+    ref = O.count(g, q, "auto", threads=THREADS)
+    assert M.tdfs_count(h, p) == ref
+    assert M.tdfs_count(h, p, M.default_opts(tau_ms=0.0, page_bytes=128)) == ref
+    gr, orig = _degree_relabel(g)
+    want = O.enumerate_sorted(gr, q, "auto")
+    want = orig[want] if want.shape[0] else want
+    want = want[np.lexsort(want.T[::-1])]
+    t, total, ovf = M.tdfs_enumerate(h, p, max(ref, 1))
+    assert total == ref and not ovf
+    t = t[np.lexsort(t.T[::-1])]
+    assert np.array_equal(t, want)
+    h.free()
+
+
 def test_enumerate_overflow_keeps_exact_total():
     g = T.rmat(10, 8, 7)
     q = T.query("triangle")
