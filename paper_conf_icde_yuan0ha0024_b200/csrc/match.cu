@@ -1439,6 +1439,22 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     cudaEventRecord(ev0, st);
   }
   KernelFn fn = pick_kernel(mode, want_stats);
+  {
+    // L1/shared split: ask for just the shared memory this launch's resident blocks need, so the rest of
+    // the 256 KB stays L1 (the hub-bitmap and adjacency probes are L1/L2 gathers).  The carveout is a
+    // sticky per-function hint: without it a launch inherits the split of an earlier, larger launch.
+    int dev = g->device, smem_sm = 0, reserved = 0;
+    cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+    cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev);
+    int sms = 1;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const long long per_sm_blocks = (L.blocks + sms - 1) / sms;
+    const long long need = per_sm_blocks * ((long long)smem_bytes(L.wpb, L.fcap) + reserved);
+    if (smem_sm > 0) {
+      const int pct = (int)std::min<long long>(100, (need * 100 + smem_sm - 1) / smem_sm);
+      cudaFuncSetAttribute(reinterpret_cast<const void*>(fn), cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+    }
+  }
   fn<<<L.blocks, L.wpb * 32, smem_bytes(L.wpb, L.fcap), st>>>(P);
   if ((e = cudaGetLastError()) != cudaSuccess) {
     cudaFree(d_trace);
