@@ -61,6 +61,8 @@ def parse():
     ap.add_argument("--hub-bitmap-mb", type=int, default=0, help="hub bitmap budget (0 = library default)")
     ap.add_argument("--degree-order", action="store_true",
                     help="load with TDFS_GRAPH_DEGREE_ORDER (symmetry breaking by degree rank, DESIGN.md R35)")
+    ap.add_argument("--also-degree-order", type=int, default=1,
+                    help="1: also time the queries on the degree-ordered graph (reported under degree_order)")
     ap.add_argument("--no-stats", action="store_true",
                     help="skip the instrumented run (no roofline bytes): long configs-3..5 queries")
     return ap.parse_args()
@@ -440,6 +442,35 @@ def run_ours(a):
                "includes": f"tdfs_load_graph (H2D of pinned CSR, src array, hub bitmaps), tdfs_plan_query x{len(qs)}, "
                            f"tdfs_count x{len(qs)}, checked reduce + D2H of the counts"}
 
+    # the same queries on the degree-ordered graph (TDFS_GRAPH_DEGREE_ORDER, R35): same counts,
+    # symmetry broken by degree rank -- reported next to the headline (which stays the paper's id order)
+    deg = None
+    if a.also_degree_order and not a.degree_order and cursors is None:
+        hd = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes, degree_order=True)
+        dws_bytes = max(M.tdfs_workspace_bytes(hd, p, o) for p, o in zip(plans, qopts))
+        dws = ws if dws_bytes <= ws.numel() else torch.empty(dws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
+        dc = torch.zeros(len(qs), dtype=torch.int64, device=f"cuda:{dev}")
+        dq = [[] for _ in qs]
+        for s in range(a.warmup + a.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            for i, p in enumerate(plans):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                M.tdfs_count(hd, p, qopts[i], workspace=dws, stream=stream, d_count=dc[i:i + 1], sync=False)
+                e1.record(stream)
+                torch.cuda.synchronize()
+                if s >= a.warmup:
+                    dq[i].append(e0.elapsed_time(e1))
+            dcounts = D.reduce_counts(dc.clone()).cpu().tolist()
+            if dcounts != counts:
+                raise RuntimeError(f"degree-ordered counts differ: {dcounts} vs {counts}")
+        dtot = sum(sum(x) for x in dq) / a.steps
+        deg = {"ms_per_step": dtot, "value": matches_per_step / (dtot / 1000.0), "unit": UNIT,
+               "counts": "equal to the id-order counts (checked every step)",
+               "per_query_ms": {q.name: sum(dq[i]) / a.steps for i, q in enumerate(qs)}}
+        hd.free()
+
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         cpu = cpu_baseline(g, qs, a.cpu_sample_world)
@@ -485,6 +516,7 @@ def run_ours(a):
             "e2e": e2e,
             "gpu_launches": 4 * len(qs) * a.steps,
             "clocks": clk,
+            "degree_order": deg,
         }
         print(json.dumps(line), flush=True)
     if cursors is not None:

@@ -163,6 +163,9 @@ void tdfs_free_plan(tdfs_plan* p);
 #define TDFS_SHARD_DEGREE_BALANCED 1  /* heavy roots (cost = sum of neighbour degrees > total/(64 W)) dealt by
                                          edge round-robin; the other roots dealt whole in snake order of
                                          decreasing cost (R31) */
+#define TDFS_SHARD_BLOCKED 2          /* blocks of 1024 consecutive directed edges dealt round-robin: block b ->
+                                         rank b mod W (keeps a root's edges on one GPU; R36) */
+#define TDFS_SHARD_BLOCK_EDGES 1024
 
 typedef struct {
   int64_t tau_ns;              /* timeout tau; default 10 ms;

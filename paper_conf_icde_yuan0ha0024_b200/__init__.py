@@ -50,6 +50,8 @@ TDFS_RUN_ARRAY_STACKS = 128
 TDFS_RUN_NO_RANGE_TASKS = 256
 TDFS_SHARD_ROUND_ROBIN = 0
 TDFS_SHARD_DEGREE_BALANCED = 1
+TDFS_SHARD_BLOCKED = 2
+TDFS_SHARD_BLOCK_EDGES = 1024
 TDFS_COUNT_INVALID = (1 << 64) - 1
 
 

@@ -162,6 +162,8 @@ struct KParams {
   uint32_t reused_mask;        // bit d: a later position / the leaf set reuses C(d) (range tasks then build it whole)
   // initial edge tasks: j -> directed edge task_edges[j] (shard list) or shard_rank + j * shard_world
   const int32_t* task_edges;   // nullptr = arithmetic shard
+  int32_t shard_block;         // arithmetic shard: 0 = edge round-robin (e = rank + j W), else blocks of this many
+                               // consecutive edges dealt round-robin (TDFS_SHARD_BLOCKED)
   unsigned long long* gcursor; // chunk cursor: this job's counter, or a cross-rank shared one (NEXT-3)
   int32_t gshared;             // gcursor is shared across ranks / devices: system-scope atomics
   // hub bitmaps (nullptr when off)

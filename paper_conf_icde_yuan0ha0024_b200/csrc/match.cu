@@ -942,8 +942,15 @@ __device__ bool run_chunk(const KParams& P, Ctx<STATS>& c, const Queue& q, long 
     int v0 = 0, v1 = 0;
     bool ok = inr;
     if (inr) {
-      const long long e = P.task_edges ? (long long)__ldg(P.task_edges + j)
-                                       : (long long)P.shard_rank + j * (long long)P.shard_world;
+      long long e;
+      if (P.task_edges) {
+        e = (long long)__ldg(P.task_edges + j);
+      } else if (P.shard_block) {  // j-th edge of this rank's blocks: block ordinal j / B -> global block
+        const long long ob = j / P.shard_block;
+        e = (ob * P.shard_world + P.shard_rank) * P.shard_block + (j - ob * P.shard_block);
+      } else {
+        e = (long long)P.shard_rank + j * (long long)P.shard_world;
+      }
       v0 = __ldg(P.src + e);
       v1 = __ldg(P.adj + e);
       if (pl.edge_cons == 1) ok = v0 < v1;
@@ -1242,7 +1249,8 @@ int resolve_layout(const Graph* g, const Plan* p, const tdfs_run_opts* o, WsLayo
   L->wpb = o->warps_per_block > 0 ? o->warps_per_block : 4;
   if (L->wpb > kBlockThreads / 32)  // the kernel's __launch_bounds__
     return fail(TDFS_E_INVALID_ARG, "opts.warps_per_block must be <= " + std::to_string(kBlockThreads / 32));
-  if (o->shard_policy != TDFS_SHARD_ROUND_ROBIN && o->shard_policy != TDFS_SHARD_DEGREE_BALANCED)
+  if (o->shard_policy != TDFS_SHARD_ROUND_ROBIN && o->shard_policy != TDFS_SHARD_DEGREE_BALANCED &&
+      o->shard_policy != TDFS_SHARD_BLOCKED)
     return fail(TDFS_E_INVALID_ARG, "opts.shard_policy");
   if (o->reserved_ != 0) return fail(TDFS_E_INVALID_ARG, "opts.reserved_ must be 0");
   if (o->shared_cursor && (reinterpret_cast<uintptr_t>(o->shared_cursor) & 7u))
@@ -1366,6 +1374,14 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
     P.n_tasks = g->nnz;
     P.gcursor = reinterpret_cast<unsigned long long*>(o->shared_cursor);
     P.gshared = 1;
+  } else if (o->shard_world > 1 && o->shard_policy == TDFS_SHARD_BLOCKED) {
+    // blocks b = rank, rank + W, ... of B edges; the last block of the graph may be partial
+    const long long B = TDFS_SHARD_BLOCK_EDGES, nb = (g->nnz + B - 1) / B, W = o->shard_world, r = o->shard_rank;
+    const long long mine = nb > r ? (nb - r + W - 1) / W : 0;
+    long long nt = mine * B;
+    if (mine > 0 && (r + (mine - 1) * W) == nb - 1) nt -= nb * B - g->nnz;  // this rank owns the partial block
+    P.n_tasks = nt;
+    P.shard_block = (int32_t)B;
   } else if (o->shard_world > 1 && o->shard_policy == TDFS_SHARD_DEGREE_BALANCED) {
     int64_t nt = 0;
     if ((rc = shard_task_list(g, o->shard_rank, o->shard_world, o->shard_policy, &P.task_edges, &nt)) != TDFS_OK)

@@ -31,6 +31,10 @@ int partition_owner(int64_t n, int64_t nnz, const int64_t* offs, const int32_t* 
     for (int64_t e = 0; e < nnz; e++) owner[e] = (int32_t)(e % world);
     return TDFS_OK;
   }
+  if (policy == TDFS_SHARD_BLOCKED) {
+    for (int64_t e = 0; e < nnz; e++) owner[e] = (int32_t)((e / TDFS_SHARD_BLOCK_EDGES) % world);
+    return TDFS_OK;
+  }
   if (policy != TDFS_SHARD_DEGREE_BALANCED) return fail(TDFS_E_INVALID_ARG, "partition: unknown policy");
   if (nnz >= (int64_t)INT32_MAX) return fail(TDFS_E_INVALID_ARG, "partition: nnz >= 2^31 (degree-balanced lists are int32)");
   if (offs[0] != 0 || offs[n] != nnz) return fail(TDFS_E_INVALID_ARG, "partition: offs[0] != 0 or offs[n] != nnz");

@@ -97,6 +97,14 @@ def test_partition_degree_balanced(world):
     assert load.max() <= 1.05 * load.mean(), load
 
 
+@pytest.mark.parametrize("world", [1, 3, 8])
+def test_partition_blocked(world):
+    """TDFS_SHARD_BLOCKED: blocks of 1024 consecutive directed edges dealt round-robin (R36)."""
+    offs, adj = _csr(T.rmat(11, 8, 2))
+    own = M.tdfs_partition_edges(offs, adj, world, M.TDFS_SHARD_BLOCKED)
+    assert np.array_equal(own, (np.arange(adj.shape[0]) // M.TDFS_SHARD_BLOCK_EDGES) % world)
+
+
 def test_partition_errors():
     offs, adj = _csr(T.rmat(6, 4, 1))
     with pytest.raises(M.TdfsError):

@@ -40,6 +40,7 @@ def _worker(rank, world, port, out):
         p = M.plan_from_query(T.query(name))
         o = M.default_opts(tau_ms=1.0, chunk=2)
         res[name] = (D.count_sharded(h, p, o), D.count_sharded(h, p, o, policy=M.TDFS_SHARD_DEGREE_BALANCED),
+                     D.count_sharded(h, p, o, policy=M.TDFS_SHARD_BLOCKED),
                      D.count_balanced(h, p, cur, o), D.count_balanced(h, p, cur, o))
         assert o.shard_world == 1 and o.shared_cursor is None  # caller's opts untouched
     cur.close()
@@ -57,4 +58,4 @@ def test_two_ranks_on_one_gpu_sharded_and_shared_cursor():
     for name in NAMES:
         ref = O.count(g, T.query(name), "auto", threads=8)
         for r in range(world):
-            assert out[r][name] == (ref, ref, ref, ref), (name, r, out[r][name], ref)
+            assert out[r][name] == (ref,) * 5, (name, r, out[r][name], ref)

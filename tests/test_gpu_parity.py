@@ -346,21 +346,23 @@ def test_shard_sum():
     for name in ["triangle", "diamond", "house"]:
         q = T.query(name)
         ref = oracle_count("r10", q, "auto")
-        for pol in (M.TDFS_SHARD_ROUND_ROBIN, M.TDFS_SHARD_DEGREE_BALANCED):
+        for pol in (M.TDFS_SHARD_ROUND_ROBIN, M.TDFS_SHARD_DEGREE_BALANCED, M.TDFS_SHARD_BLOCKED):
             for W in (2, 3, 8):
                 assert sum(U.count(rmat12, q, "auto", shard_rank=r, shard_world=W, shard_policy=pol)
                            for r in range(W)) == ref, (name, pol, W)
 
 
-def test_degree_balanced_shards_match_oracle_on_owned_edges():
-    """A degree-balanced shard counts exactly the matches whose root edge it owns: the oracle
-    restricted to one round-robin shard of W' = nnz (a single edge) summed over the edges
-    tdfs_partition_edges gives rank r equals the kernel's rank-r count (small graph)."""
+@pytest.mark.parametrize("policy", [1, 2])
+def test_partitioned_shards_match_oracle_on_owned_edges(policy):
+    """A degree-balanced (1) or blocked (2) shard counts exactly the matches whose root edge it owns:
+    the oracle restricted to one round-robin shard of W' = nnz (a single edge) summed over the edges
+    tdfs_partition_edges gives rank r equals the kernel's rank-r count (small graph, several blocks)."""
     import paper_conf_icde_yuan0ha0024_b200 as M
     g = T.rmat(8, 6, 5)
     offs, adj = T.to_csr(g)
+    assert adj.shape[0] > 2 * M.TDFS_SHARD_BLOCK_EDGES
     W = 3
-    own = M.tdfs_partition_edges(offs, adj, W, M.TDFS_SHARD_DEGREE_BALANCED)
+    own = M.tdfs_partition_edges(offs, adj, W, policy)
     q = T.query("diamond")
     order = O.oracle_order(q)
     nnz = adj.shape[0]
@@ -368,8 +370,7 @@ def test_degree_balanced_shards_match_oracle_on_owned_edges():
     per_edge = [O.count(og, q, "auto", order=order, shard=(e, nnz)) for e in range(nnz)]
     for r in range(W):
         want = sum(c for c, o in zip(per_edge, own) if o == r)
-        got = U.count(g, q, "auto", order=order, shard_rank=r, shard_world=W,
-                      shard_policy=M.TDFS_SHARD_DEGREE_BALANCED)
+        got = U.count(g, q, "auto", order=order, shard_rank=r, shard_world=W, shard_policy=policy)
         assert got == want, r
 
 
