@@ -29,7 +29,10 @@ int fail(int status, const std::string& msg);  // sets the detail, returns statu
 // |F ∩ N(S[k-2])| (or |F| minus S[k-2]) under the S[k-2]-dependent window.
 constexpr int kVF = kMaxK;
 constexpr int kBlockThreads = 128;  // matching-kernel block size (its __launch_bounds__)
-constexpr int kLeafStage = 512;  // shared-memory ids per warp for a materialised leaf set F (at most)
+#ifndef TDFS_LEAF_STAGE_MAX  // build-time constant (experiments build variants with -D)
+#define TDFS_LEAF_STAGE_MAX 512
+#endif
+constexpr int kLeafStage = TDFS_LEAF_STAGE_MAX;  // shared-memory ids per warp for a materialised leaf set F (at most)
 // Hub bitmaps (graph.cu): vertices of degree >= kHubMinDeg, highest first, within the budget
 constexpr int64_t kHubMinDeg = 256;
 constexpr int64_t kHubBudgetDefault = 256ll << 20;

@@ -1,0 +1,8 @@
+#!/bin/bash
+export PYTHONPATH=$PWD
+P=scripts/configs_probe.py
+timeout 300 python $P 4 prism 512 0 0 10 0 stats
+timeout 300 python $P 4 prism 64 0 0 -1 0 stats
+timeout 300 python $P 4 prism 64 0,1 0 10 0 stats
+timeout 300 python $P 4 w5 64 0 0 10 0 stats
+timeout 300 python $P 4 prism 1 0 0 10 0 stats

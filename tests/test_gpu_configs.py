@@ -34,7 +34,8 @@ def _query(cfg, name):
     return T.labeled_query(name, 8) if cfg == 4 else T.query(name)
 
 
-CASES = [(cfg, name) for cfg in (3, 4, 5) for name in T.CONFIG_QUERIES[cfg]]
+CASES = [(cfg, name) for cfg in (3, 4, 5) for name in T.CONFIG_QUERIES[cfg]] + \
+    [(cfg, name) for cfg in (3, 4, 5) for name in T.BENCH_QUERIES[cfg] if name not in T.CONFIG_QUERIES[cfg]]
 
 
 @pytest.mark.parametrize("cfg,name", CASES)
@@ -63,3 +64,14 @@ def test_config_planner_order_equals_oracle_order_full_count(cfg, name):
     a = U.count(g, q, "auto")
     b = U.count(g, q, "auto", order=O.oracle_order(q))
     assert a == b > 0, (cfg, name, a, b)
+
+
+def test_config3_k5_full_count_equals_oracle_golden():
+    """The C3 bench query in bench.py's launch configuration (planner order, tau = 10 ms, chunk 1)
+    equals the oracle's full-graph count (tests/golden/c3_counts.txt, scripts/golden_counts.py)."""
+    import paper_conf_icde_yuan0ha0024_b200 as M
+    from tests import golden_io as G
+    gold = int(G.read("c3_counts.txt")["k5"].split()[0])
+    g = _cfg(3)[0]
+    h = U.load(g)
+    assert M.tdfs_count(h, M.plan_from_query(T.query("k5")), M.default_opts(chunk=1)) == gold
