@@ -39,6 +39,12 @@ METRIC = "matches/sec & time-to-count per query at 1/2/4/8 B200; HBM GB/s fracti
 UNIT = "matches/s"
 
 
+# timeout tau per config (PAPER.md:486-518 tunes tau per dataset; 10 ms is the paper's choice): measured on
+# one B200 -- C4 prism/w5 1 ms (33.0 / 12.7 s vs 36.6 / 14.0 s at 10 ms), C5 k4 100 ms (1/16 shard 2.66 s vs
+# 3.85 s at 10 ms, 5.31 s at 1 ms); profiles/c4_splitting_diag_r02.txt, profiles/c45_r02o.log
+TAU_DEFAULT_MS = {4: 1.0, 5: 100.0}
+
+
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -46,7 +52,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", type=int, default=2)
-    ap.add_argument("--tau-ms", type=float, default=10.0)
+    ap.add_argument("--tau-ms", type=float, default=None,
+                    help="timeout tau (ms, < 0 = none); default per config: TAU_DEFAULT_MS (measured sweeps, DESIGN.md 10)")
     ap.add_argument("--chunk", type=int, default=1,
                     help="initial edge tasks per cursor grab (ABI default 8 = the paper's; 1 measured best on config 2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -276,6 +283,8 @@ def run_ours(a):
     t_plan0 = time.perf_counter()
     plans = [M.plan_from_query(q) for q in qs]
     plan_s = time.perf_counter() - t_plan0
+    if a.tau_ms is None:
+        a.tau_ms = TAU_DEFAULT_MS.get(a.config, 10.0)
     tau = None if a.tau_ms < 0 else a.tau_ms
     cursors = D.SharedCursorGroup(dev) if (world > 1 and a.shared_cursor) else None
     # per query: k = 3 jobs are one intersection per edge task, so they keep the paper's chunk of 8
@@ -392,11 +401,17 @@ def run_ours(a):
         nq = ncu["per_query"][qs[dom].name]
         traffic = nq.get("dram_bytes")
         if nq.get("lts_bytes") is not None:
+            dur = nq["duration_ms"] / 1000.0
             l2 = {"lts_t_bytes": nq["lts_bytes"], "ncu_duration_ms": nq.get("duration_ms"),
-                  "achieved_GBps": nq["lts_bytes"] / (nq["duration_ms"] / 1000.0) / 1e9,
+                  "achieved_GBps": nq["lts_bytes"] / dur / 1e9,
                   "peak_GBps": ncu.get("l2_peak_gbs"), "l2_hit_rate": nq.get("l2_hit"),
-                  "frac": (nq["lts_bytes"] / (nq["duration_ms"] / 1000.0) / 1e9) / ncu["l2_peak_gbs"]
-                  if ncu.get("l2_peak_gbs") else None}
+                  "frac": (nq["lts_bytes"] / dur / 1e9) / ncu["l2_peak_gbs"] if ncu.get("l2_peak_gbs") else None}
+            if nq.get("lts_read_sectors_sm") is not None and ncu.get("l2_random_sectors_per_ns"):
+                # the kernel's reads are scattered probes: compare the L2->SM sector rate with the measured
+                # rate of random 32-B sector reads from an L2-resident buffer (scripts/l2_peak.cu)
+                rate = nq["lts_read_sectors_sm"] / dur / 1e9
+                l2.update({"read_sectors_per_ns": rate, "peak_random_sectors_per_ns": ncu["l2_random_sectors_per_ns"],
+                           "frac_random_sectors": rate / ncu["l2_random_sectors_per_ns"]})
 
     # e2e through the public API with host buffers: H2D of the CSR from pinned memory,
     # load, plan, the counts, D2H of the counts -- every step

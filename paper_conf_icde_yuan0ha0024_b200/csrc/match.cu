@@ -531,7 +531,19 @@ __device__ __forceinline__ void lower_bound4(const int* L, int lo, int n, int v0
   r3 += L[r3] < v3;
 }
 
-__device__ __forceinline__ unsigned bit_of(const uint32_t* row, int v) { return (__ldg(row + (v >> 5)) >> (v & 31)) & 1u; }
+// L2 residency hints (north_star; prims.cuh ldg_hint), a build-time experiment, off by default: measured
+// with no gain.  Bit 0: hub-bitmap probes evict_last; bit 1: stream-B N(x) loads
+// evict_first; bit 2 (with bit 1): N(x) of a hub leaf evict_last instead.
+#ifndef TDFS_L2HINT
+#define TDFS_L2HINT 0
+#endif
+__device__ __forceinline__ unsigned bit_of(const uint32_t* row, int v) {
+#if TDFS_L2HINT & 1
+  return (ldg_hint(row + (v >> 5), l2_evict_last()) >> (v & 31)) & 1u;
+#else
+  return (__ldg(row + (v >> 5)) >> (v & 31)) & 1u;
+#endif
+}
 
 // A whole batch of nb <= 32 staged leaves at once: lane j
 // holds leaf x_j = S[k-2] and N(x_j)'s metadata.  The count is only summed, so the batch's
@@ -688,6 +700,9 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
     const int4* const adj4 = reinterpret_cast<const int4*>(P.adj);
     const uint32_t* const frow = fr.hid >= 0 ? P.hub_bits + (long long)fr.hid * P.hub_words : nullptr;
     int j = -1, jn = 0, pj = 0, loj = 0, hij = 0, fminj = 0, fmaxj = 0;
+#if TDFS_L2HINT & 4
+    int hidB = -1;
+#endif
     long long g0 = 0, sj = 0, ej = 0;
     for (int base = 0; base < tot; base += 32) {
       const int idx = base + lane;
@@ -699,6 +714,9 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
           pj = pre[j];
           const LeafMeta e = meta[j];
           loj = e.lo; hij = e.hi;
+#if TDFS_L2HINT & 4
+          hidB = e.hid;
+#endif
           sj = e.b0 + e.s;
           ej = e.b0 + e.e;
           g0 = sj >> 2;
@@ -706,7 +724,15 @@ __device__ long long leaf_batch(const KParams& P, Ctx<STATS>& c, const FRef& fr,
           fmaxj = F[hij - 1];
         }
         const long long g = g0 + idx - pj;
+#if TDFS_L2HINT & 2
+#if TDFS_L2HINT & 4
+        q = ldg_hint4(adj4 + g, hidB >= 0 ? l2_evict_last() : l2_evict_first());
+#else
+        q = ldg_hint4(adj4 + g, l2_evict_first());
+#endif
+#else
         q = __ldg(adj4 + g);
+#endif
         const long long i0 = g << 2;
         k0 = i0 >= sj && i0 < ej && q.x >= fminj && q.x <= fmaxj;
         k1 = i0 + 1 >= sj && i0 + 1 < ej && q.y >= fminj && q.y <= fmaxj;
@@ -1359,7 +1385,12 @@ int launch_job(const Graph* g, const Plan* p, const tdfs_run_opts* o, void* ws, 
   if (!(o->flags & TDFS_RUN_NO_RANGE_TASKS)) {
     for (int d = 2; d <= std::min(kMaxRangeLevel, P.plan.k - 2); d++) {
       const bool leaf_level_reused = d == P.plan.k - 2 && ((P.reused_mask >> d) & 1u) && P.plan.lf_var;
+#ifdef TDFS_RANGE_LEAF_REUSED  // build-time experiment: range tasks also for a reused leaf-parent level
+      if (true) P.range_mask |= 1u << d;
+      (void)leaf_level_reused;
+#else
       if (!leaf_level_reused) P.range_mask |= 1u << d;
+#endif
     }
     P.split_mask |= P.range_mask;  // deeper levels split only into range tasks
   }

@@ -47,6 +47,36 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   return m;
 }
 
+// L2 residency hints (north_star "Blackwell L2 residency hints for hub adjacency lists"): a
+// cache policy built by createpolicy and attached to a read-only load with .L2::cache_hint.
+// evict_last keeps the line in L2 ahead of normal lines; evict_first lets it go first.
+__device__ __forceinline__ unsigned long long l2_evict_last() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ unsigned long long l2_evict_first() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ unsigned ldg_hint(const unsigned* a, unsigned long long pol) {
+  unsigned v;
+  asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int ldg_hint(const int* a, unsigned long long pol) {
+  int v;
+  asm("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int4 ldg_hint4(const int4* a, unsigned long long pol) {
+  int4 v;
+  asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a), "l"(pol));
+  return v;
+}
+
 __device__ __forceinline__ unsigned long long* ctr(const KParams& P, int i) { return P.ctr + i * kCounterStride; }
 
 __device__ __forceinline__ int read_error(const KParams& P) {

@@ -20,7 +20,10 @@ want = {"duration_ms": ("gpu__time_duration.sum", 1e-6), "dram_read": ("dram__by
         "inst_executed": ("smsp__inst_executed.sum", 1), "registers": ("launch__registers_per_thread", 1),
         "threads_per_inst": ("smsp__thread_inst_executed_per_inst_executed.ratio", 1),
         "local_load_sectors": ("l1tex__t_sectors_pipe_lsu_mem_local_op_ld.sum", 1),
-        "local_store_sectors": ("l1tex__t_sectors_pipe_lsu_mem_local_op_st.sum", 1)}
+        "local_store_sectors": ("l1tex__t_sectors_pipe_lsu_mem_local_op_st.sum", 1),
+        "lts_sectors": ("lts__t_sectors.sum", 1),
+        "lts_read_sectors_sm": ("lts__t_sectors_srcunit_tex_op_read.sum", 1),
+        "lts_throughput_pct": ("lts__throughput.avg.pct_of_peak_sustained_elapsed", 1)}
 scale_units = {"ns": 1, "us": 1e3, "ms": 1e6, "s": 1e9, "byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9,
                "Tbyte": 1e12}
 per = {}
@@ -45,15 +48,19 @@ for q in qs:
         v *= scale_units.get(units[col[m]], 1)
         d[k] = v * sc
     d["dram_bytes"] = d.get("dram_read", 0) + d.get("dram_write", 0)
+    if "lts_bytes" not in d and "lts_sectors" in d:
+        d["lts_bytes"] = 32.0 * d["lts_sectors"]
     per[q] = d
-l2 = None
+l2, l2r = None, None
 p = f"gpurun_out/l2_peak_{tag}.json"
 if os.path.exists(p):
-    l2 = json.load(open(p))["l2_read_peak_gbs"]
+    lj = json.load(open(p))
+    l2 = lj["l2_read_peak_gbs"]
+    l2r = lj.get("l2_random_sectors_per_ns")
 out = {"round": tag, "config": cfg, "source_hash": kernel_source_hash(), "kernel": "tdfs_kernel<0,0> (count, no stats)",
        "source": "ncu --set full --clock-control none --import-source on, one timed launch per query "
                  "(bench.py --steps 1 --warmup 0 --queries q; -s 1 skips the STATS launch)",
-       "l2_peak_gbs": l2, "per_query": per}
+       "l2_peak_gbs": l2, "l2_random_sectors_per_ns": l2r, "per_query": per}
 json.dump(out, open(f"gpurun_out/ncu_full_summary_{tag}.json", "w"), indent=1)
 for q, d in per.items():
     print(q, {k: round(v, 4) if isinstance(v, float) else v for k, v in d.items()})
