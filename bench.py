@@ -460,7 +460,8 @@ def run_ours(a):
     # the same queries on the degree-ordered graph (TDFS_GRAPH_DEGREE_ORDER, R35): same counts,
     # symmetry broken by degree rank -- reported next to the headline (which stays the paper's id order)
     deg = None
-    if a.also_degree_order and not a.degree_order and cursors is None:
+    # (a profiling shard of the renumbered graph holds other root edges: compare only whole-graph counts)
+    if a.also_degree_order and not a.degree_order and cursors is None and a.profile_shard_world == 1:
         hd = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes, degree_order=True)
         dws_bytes = max(M.tdfs_workspace_bytes(hd, p, o) for p, o in zip(plans, qopts))
         dws = ws if dws_bytes <= ws.numel() else torch.empty(dws_bytes, dtype=torch.uint8, device=f"cuda:{dev}")
