@@ -279,7 +279,8 @@ def test_hub_bitmaps_do_not_change_results():
     import paper_conf_icde_yuan0ha0024_b200 as M
     g = T.rmat(12, 24, 5)
     assert int(np.bincount(g.edges.reshape(-1)).max()) >= 256
-    for name in ["triangle", "k4"]:
+    # c4: referenced leaf sets F of hubs probed by bitmap against hub leaves (flat leaf batches, streams A/B)
+    for name in ["triangle", "k4", "c4"]:
         q = T.query(name)
         ref = O.count(g, q, "auto", threads=THREADS)
         assert U.count(g, q, "auto") == ref
