@@ -43,6 +43,10 @@ UNIT = "matches/s"
 # one B200 -- C4 prism/w5 1 ms (33.0 / 12.7 s vs 36.6 / 14.0 s at 10 ms), C5 k4 100 ms (1/16 shard 2.66 s vs
 # 3.85 s at 10 ms, 5.31 s at 1 ms); profiles/c4_splitting_diag_r02.txt, profiles/c45_r02o.log
 TAU_DEFAULT_MS = {4: 1.0, 5: 100.0}
+# hub-bitmap budget per config (MB; library default 256 MB): measured on one B200 (profiles/hub_budget_r02s.log,
+# 256 MB / 1 / 4 / 16 GB): C5 k4 1/16 shard 2.66 / 2.14 / 2.20 / 2.46 s, C4 prism 1/64 0.79 / 0.69 / 0.76 / 0.74 s,
+# w5 flat; C3 c5 16.5 / 18.8 s (more bitmaps than the lists they replace thrash L2), C3 k5 flat
+HUB_MB_DEFAULT = {4: 1024, 5: 1024}
 
 
 def parse():
@@ -65,7 +69,8 @@ def parse():
     ap.add_argument("--flags", type=int, default=0, help="tdfs_run_opts.flags (ablations)")
     ap.add_argument("--shard-policy", type=int, default=0, help="N > 1: 0 round-robin (paper), 1 degree-balanced")
     ap.add_argument("--shared-cursor", action="store_true", help="N > 1: cross-GPU shared chunk cursor (NEXT-3)")
-    ap.add_argument("--hub-bitmap-mb", type=int, default=0, help="hub bitmap budget (0 = library default)")
+    ap.add_argument("--hub-bitmap-mb", type=int, default=None,
+                    help="hub bitmap budget (0 = library default); default per config: HUB_MB_DEFAULT")
     ap.add_argument("--degree-order", action="store_true",
                     help="load with TDFS_GRAPH_DEGREE_ORDER (symmetry breaking by degree rank, DESIGN.md R35)")
     ap.add_argument("--also-degree-order", type=int, default=1,
@@ -274,6 +279,8 @@ def run_ours(a):
     if a.queries:
         keep = set(a.queries.split(","))
         qs = [q for q in qs if q.name in keep or q.name.replace("_lab", "") in keep]
+    if a.hub_bitmap_mb is None:
+        a.hub_bitmap_mb = HUB_MB_DEFAULT.get(a.config, 0)
     hub_bytes = a.hub_bitmap_mb << 20
     t_load0 = time.perf_counter()
     h = M.tdfs_load_edges(g.n, g.edges, g.labels, device=dev, hub_bitmap_bytes=hub_bytes, degree_order=a.degree_order)
@@ -514,7 +521,7 @@ def run_ours(a):
                        "queries": [q.name for q in qs],
                        "constraints": "full symmetry breaking (stabilizer chain)" +
                                       (" on degree ranks (TDFS_GRAPH_DEGREE_ORDER)" if a.degree_order else " on vertex ids"),
-                       "tau_ms": a.tau_ms, "chunk": {"k3": 8, "k>=4": a.chunk},
+                       "tau_ms": a.tau_ms, "hub_bitmap_mb": a.hub_bitmap_mb or 256, "chunk": {"k3": 8, "k>=4": a.chunk},
                        "parallelism": f"shard{world}" + ("-shared-cursor" if cursors is not None else
                                                          f"-policy{a.shard_policy}"),
                        "l2": "flushed (256 MB write) before every timed step", "load_s": load_s, "plan_s": plan_s,
