@@ -15,6 +15,11 @@ PAPER.md:522, or --shard-policy 1 degree-balanced, R31; or --shared-cu
 take edge chunks from one cursor in rank 0's HBM, NEXT-3) and one NCCL all-reduce of
 {count, failed} sums the counts -- total work is fixed: "strong".
 
+--config 3/4/5: the gated query sets of tdfs_inputs.BENCH_QUERIES with the per-config timeout tau
+(TAU_DEFAULT_MS) and hub-bitmap budget (HUB_MB_DEFAULT) that this repo's sweeps found best (R37, section 10).
+The roofline object reports the dominant launch: R32 algorithmic bytes / its CUDA-event time against the measured
+HBM peak, the same-source ncu DRAM traffic, and (config 2) its L2 sector rate against the measured L2 peaks.
+
 After timing, the counts are checked against the oracle goldens of the config
 (tests/golden/c<cfg>_counts.txt, written by scripts/golden_counts.py from oracle/ only) when
 the file has them; a mismatch or a failed job (TDFS_COUNT_INVALID) aborts the run.
