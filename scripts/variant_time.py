@@ -24,7 +24,8 @@ print(f"lib {M.LIB_PATH} hub_mb {hub_mb} degree_order {degree_order}", flush=Tru
 for name in qn:
     q = T.labeled_query(name, 8) if cfg == 4 else T.query(name)
     p = M.plan_from_query(q)
-    o = M.default_opts(chunk=8 if q.k <= 3 else 1, shard_world=W, tau_ms=float(os.environ.get("TAU", "10")))
+    o = M.default_opts(chunk=8 if q.k <= 3 else int(os.environ.get("CHUNK", "1")), shard_world=W,
+                       tau_ms=float(os.environ.get("TAU", "10")))
     ts = []
     for r in range(reps + 1):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
