@@ -47,7 +47,8 @@ UNIT = "matches/s"
 # timeout tau per config (PAPER.md:486-518 tunes tau per dataset; 10 ms is the paper's choice): measured on
 # one B200 -- C4 prism/w5 1 ms (33.0 / 12.7 s vs 36.6 / 14.0 s at 10 ms), C5 k4 100 ms (1/16 shard 2.66 s vs
 # 3.85 s at 10 ms, 5.31 s at 1 ms); profiles/c4_splitting_diag_r02.txt, profiles/c45_r02o.log
-TAU_DEFAULT_MS = {4: 1.0, 5: 100.0}
+# C3 k5 100 ms (723 vs 868 ms at 10 ms, profiles/tau_r02aa.log); C2's five-query step is flat over 10-100 ms
+TAU_DEFAULT_MS = {3: 100.0, 4: 1.0, 5: 100.0}
 # hub-bitmap budget per config (MB; library default 256 MB): measured on one B200 (profiles/hub_budget_r02s.log,
 # 256 MB / 1 / 4 / 16 GB): C5 k4 1/16 shard 2.66 / 2.14 / 2.20 / 2.46 s, C4 prism 1/64 0.79 / 0.69 / 0.76 / 0.74 s,
 # w5 flat; C3 c5 16.5 / 18.8 s (more bitmaps than the lists they replace thrash L2), C3 k5 flat
